@@ -1,0 +1,525 @@
+// rcm_batch.cuh -- per-batch work of the batch-based RCM (one persistent thread
+// block = one worker): parent load, speculative discovery,
+// rediscovery, per-parent (valence, id) sort, output with fused reverse, and
+// batch generation with work aggregation.  Citations P:L<n> = PAPER.md line n.
+#pragma once
+#include "rcm_device.cuh"
+
+namespace rcm {
+
+// Kernel-wide parameters (passed by value to every kernel).
+struct KParams {
+  const int32_t* row_ptr;
+  const int32_t* col_idx;
+  unsigned long long* word;   // per node: owner key (hi 32) | valence (lo 32)
+  int32_t* o;                 // CM order (matrix-local ids at matrix-local positions)
+  int32_t* perm;              // output, new -> old
+  int32_t* iperm;             // nullable, old -> new (single graph)
+  Desc* desc;                 // batch queue
+  Sig* sig;                   // per-slot signals (qcap + 1)
+  Ctl* ctl;
+  Stats* stats;
+  const Problem* chains;
+  const Problem* solos;
+  unsigned long long* spill;  // oversize scratch: [0, spill_cap) keys, [spill_cap, 2*spill_cap) temp
+  int64_t spill_cap;
+  int32_t qcap;
+  int32_t BS;                 // B_s
+  int32_t T;                  // temp elements per batch
+  int32_t flags;
+  int32_t collect_stats;
+  int32_t nblocks;
+};
+
+enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8 };
+
+// Dynamic shared memory of one worker.
+struct SmemPtrs {
+  unsigned long long* cand;   // T+1 candidate keys (valence << 32 | id); reused for prefixes
+  uint16_t* lpof;             // T local parent id of every edge slot
+  int32_t* p_v;               // BS parent ids
+  int32_t* p_rs;              // BS row start (local, add ci_base)
+  int32_t* p_eo;              // BS+1 edge-slot offsets (exclusive prefix of row lengths)
+  int32_t* p_cnt;             // BS slots used (claims) per parent
+  int32_t* p_keep;            // BS kept children per parent
+  int32_t* p_out;             // BS+1 output offsets
+};
+
+__host__ __device__ inline size_t smem_bytes(int BS, int T) {
+  return sizeof(unsigned long long) * (size_t)(T + 1) + sizeof(uint16_t) * (size_t)T + 16 +
+         sizeof(int32_t) * (size_t)(6 * BS + 2) + 64;
+}
+
+__device__ inline SmemPtrs carve_smem(unsigned char* base, int BS, int T) {
+  SmemPtrs s;
+  size_t off = 0;
+  s.cand = reinterpret_cast<unsigned long long*>(base);
+  off += sizeof(unsigned long long) * (size_t)(T + 1);
+  s.lpof = reinterpret_cast<uint16_t*>(base + off);
+  off += sizeof(uint16_t) * (size_t)T;
+  off = (off + 15) & ~size_t(15);
+  int32_t* ip = reinterpret_cast<int32_t*>(base + off);
+  s.p_v = ip;
+  s.p_rs = ip + BS;
+  s.p_eo = ip + 2 * BS;          // BS + 1
+  s.p_cnt = ip + 3 * BS + 1;
+  s.p_keep = ip + 4 * BS + 1;
+  s.p_out = ip + 5 * BS + 1;     // BS + 1
+  return s;
+}
+
+// Static shared state of one worker.
+struct ShState {
+  unsigned long long wtmp64[kWarps + 1];
+  int32_t wtmp32[kWarps + 1];
+  long long wtmpll[kWarps + 1];
+  int32_t t, o_begin, o_end, next;
+  int32_t nP, E, steal, removed;
+  int32_t s_early, s_mid, counted, aborted;
+  int32_t out_off, q_off, ovh_n, ovh_t;
+  int32_t fwd, nb, count, chain_end;
+  long long V;
+  int32_t k, written, pos, big_n;
+  unsigned long long minkey;
+  int64_t spill_base;
+  int32_t big_list[256];
+};
+
+__device__ __forceinline__ void latch_error(Ctl* ctl, int32_t code) {
+  atomicCAS(&ctl->status, 0, code);
+  atomicExch(&ctl->done, 1);
+}
+
+// ---------------------------------------------------------------- signals
+__device__ __forceinline__ uint32_t load_state(const Sig* s, uint32_t epoch) {
+  unsigned long long w = ld_acquire_u64(&s->word);
+  return (uint32_t)(w >> 32) == epoch ? (uint32_t)(w & 0xffffffffu) : S_NONE;
+}
+
+__device__ __forceinline__ void send_state(Sig* s, uint32_t epoch, uint32_t st) {
+  __threadfence();
+  st_release_u64(&s->word, ((unsigned long long)epoch << 32) | st);
+}
+
+// Busy wait with sleep back-off.  Returns the state, or S_NONE if
+// the chain was terminated (done) or the watchdog fired.
+__device__ uint32_t wait_state(const Sig* s, uint32_t epoch, uint32_t need, Ctl* ctl) {
+  uint32_t st = load_state(s, epoch);
+  if (st >= need) return st;
+  uint64_t t0 = globaltimer();
+  unsigned ns = 32;
+  for (;;) {
+    if (ld_relaxed_s32(&ctl->done)) return S_NONE;
+    __nanosleep(ns);
+    if (ns < 512) ns <<= 1;
+    st = load_state(s, epoch);
+    if (st >= need) return st;
+    if (globaltimer() - t0 > kWatchdogNs) {
+      latch_error(ctl, ST_HANG);
+      return S_NONE;
+    }
+  }
+}
+
+// ----------------------------------------------------------- parent load
+// Load the parents o[o_base + o_begin + lp], lp < nP, their row starts and the
+// exclusive prefix of their row lengths into p_eo.  If cut_T, shrink nP to the
+// longest prefix whose edge count fits T (at least one parent) -- the solo
+// worker's batch formation.  Returns nP; sh.E = edge slots.
+__device__ int load_parents(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                            int o_begin, int nP, bool cut_T) {
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
+    int v = ld_cg_s32(kp.o + P.o_base + o_begin + lp);
+    const int32_t* rp = kp.row_ptr + P.rp_base + v;
+    int rs = __ldg(rp), re = __ldg(rp + 1);
+    sm.p_v[lp] = v;
+    sm.p_rs[lp] = rs;
+    sm.p_eo[lp] = re - rs;
+  }
+  __syncthreads();
+  int E = block_scan_array<int32_t>(sm.p_eo, nP, sh.wtmp32);
+  sm.p_eo[nP] = E;   // (visible after the barrier below)
+  __syncthreads();
+  if (cut_T && E > kp.T && nP > 1) {
+    // largest nP' with p_eo[nP'] <= T (p_eo is non-decreasing); at least 1.
+    if (threadIdx.x == 0) {
+      int lo = 1, hi = nP;   // p_eo[lo] may exceed T when the first row alone is oversize
+      while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (sm.p_eo[mid] <= kp.T) lo = mid; else hi = mid - 1;
+      }
+      sh.nP = lo;
+    }
+    __syncthreads();
+    nP = sh.nP;
+    E = sm.p_eo[nP];
+  }
+  if (threadIdx.x == 0) { sh.nP = nP; sh.E = E; }
+  __syncthreads();
+  return nP;
+}
+
+// largest lp in [lo, nP) with p_eo[lp] <= e
+__device__ __forceinline__ int find_parent(const int32_t* p_eo, int lo, int nP, int e) {
+  int hi = nP - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (p_eo[mid] <= e) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+// -------------------------------------------------- speculative discovery
+// Alg. 4 discover with parent-rank keys (C-4):
+// key(p) = pos(p) + 1; m_n <- atomicMin(word[n], key); n is a candidate of p
+// iff the old owner was larger.  The valence comes back in the same 64-bit word
+// ("immediately compute the valence").  Candidates go to p's segment
+// of the scratchpad ("atomicAdd to reserve a unique spot").
+__device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                         int o_begin, int nP, int E) {
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm.p_cnt[lp] = 0;
+  __syncthreads();
+  const uint32_t kfirst = (uint32_t)o_begin + 1, klast = (uint32_t)o_begin + (uint32_t)nP;
+  int steal = 0, claims = 0;
+  int lp = 0;
+  unsigned long long* word = kp.word + P.node_base;
+  const int32_t* col = kp.col_idx + P.ci_base;
+  for (int e = threadIdx.x; e < E; e += kThreads) {
+    lp = find_parent(sm.p_eo, lp, nP, e);
+    sm.lpof[e] = (uint16_t)lp;
+    int c = __ldg(col + sm.p_rs[lp] + (e - sm.p_eo[lp]));
+    uint32_t key = kfirst + (uint32_t)lp;
+    unsigned long long w = ld_relaxed_u64(word + c);
+    if ((uint32_t)(w >> 32) > key) {
+      unsigned long long old = atomicMin(word + c, ((unsigned long long)key << 32) | (w & 0xffffffffull));
+      uint32_t ow = (uint32_t)(old >> 32);
+      if (ow > key) {
+        int slot = sm.p_eo[lp] + atomicAdd(&sm.p_cnt[lp], 1);
+        sm.cand[slot] = ((old & 0xffffffffull) << 32) | (uint32_t)c;
+        steal |= (ow <= klast);   // taken from a sibling parent of this batch
+        ++claims;
+      }
+    }
+  }
+  if (__syncthreads_or(steal) && threadIdx.x == 0) sh.steal = 1;
+  if (kp.collect_stats) {
+    int tot = block_reduce_sum<int32_t>(claims, sh.wtmp32);
+    if (threadIdx.x == 0 && tot) atomicAdd(&kp.stats->cand_spec, (unsigned long long)tot);
+  }
+  for (int i = threadIdx.x; i < nP; i += kThreads) sm.p_keep[i] = sm.p_cnt[i];
+  __syncthreads();
+}
+
+// ------------------------------------------------------------ rediscovery
+// Alg. 4 rediscover: drop n from c if a predecessor (or a sibling
+// parent with a smaller key) owns it now: keep iff owner(n) == key(p).
+// Removed candidates become kKeyMax (sorted to the end of their segment).
+__device__ int rediscover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                          int o_begin, int E) {
+  const unsigned long long* word = kp.word + P.node_base;
+  int removed = 0;
+  for (int e = threadIdx.x; e < E; e += kThreads) {
+    int lp = sm.lpof[e];
+    if (e - sm.p_eo[lp] >= sm.p_cnt[lp]) continue;
+    unsigned long long k = sm.cand[e];
+    if (k == kKeyMax) continue;
+    uint32_t c = (uint32_t)k;
+    uint32_t key = (uint32_t)o_begin + 1 + (uint32_t)lp;
+    if ((uint32_t)(ld_relaxed_u64(word + c) >> 32) != key) {
+      sm.cand[e] = kKeyMax;
+      atomicSub(&sm.p_keep[lp], 1);
+      ++removed;
+    }
+  }
+  int tot = block_reduce_sum<int32_t>(removed, sh.wtmp32);
+  if (kp.collect_stats && threadIdx.x == 0 && tot)
+    atomicAdd(&kp.stats->cand_removed, (unsigned long long)tot);
+  return tot;
+}
+
+// ------------------------------------------------------------------ sort
+// Ascending sort of keys a[0..n) with a bitonic network in which every
+// comparator places the minimum at the lower index (the "flip" formulation), so
+// virtual +inf padding beyond n needs no storage.  Executed by `nthr` threads
+// (tid = rank in the group); `sync()` is the group barrier.
+template <typename Sync>
+__device__ __forceinline__ void bitonic_sort_flip(unsigned long long* a, int n, int tid, int nthr,
+                                                  Sync sync) {
+  int N = 1;
+  while (N < n) N <<= 1;
+  for (int k = 2; k <= N; k <<= 1) {
+    // flip stage: compare i with the mirrored partner inside each k-block
+    for (int i = tid; i < N / 2; i += nthr) {
+      int blk = i / (k / 2);
+      int off = i % (k / 2);
+      int lo = blk * k + off;
+      int hi = blk * k + k - 1 - off;
+      if (hi < n) {
+        unsigned long long x = a[lo], y = a[hi];
+        if (y < x) { a[lo] = y; a[hi] = x; }
+      }
+    }
+    sync();
+    for (int j = k / 4; j > 0; j >>= 1) {
+      for (int i = tid; i < N / 2; i += nthr) {
+        int blk = i / j;
+        int off = i % j;
+        int lo = blk * 2 * j + off;
+        int hi = lo + j;
+        if (hi < n) {
+          unsigned long long x = a[lo], y = a[hi];
+          if (y < x) { a[lo] = y; a[hi] = x; }
+        }
+      }
+      sync();
+    }
+  }
+}
+
+// Sort every parent's segment cand[p_eo[lp] .. p_eo[lp] + p_cnt[lp]) by
+// (valence, id) -- Alg. 1 ln 14 "sort(c)" per parent, equivalently the
+// GPU key (local parent, valence) of P:L778-781 with the id tie-break of C-1.
+// Tiny segments: one thread (insertion sort); medium: one warp; large: block.
+__device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh, int nP) {
+  if (threadIdx.x == 0) sh.big_n = 0;
+  __syncthreads();
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
+    int n = sm.p_cnt[lp];
+    if (n <= 1) continue;
+    unsigned long long* a = sm.cand + sm.p_eo[lp];
+    if (n <= 16) {
+      for (int i = 1; i < n; ++i) {
+        unsigned long long x = a[i];
+        int j = i - 1;
+        while (j >= 0 && a[j] > x) { a[j + 1] = a[j]; --j; }
+        a[j + 1] = x;
+      }
+    } else {
+      int idx = atomicAdd(&sh.big_n, 1);
+      if (idx < 256) sh.big_list[idx] = lp;
+    }
+  }
+  __syncthreads();
+  int nbig = sh.big_n;
+  if (nbig == 0) return;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (nbig <= 256) {
+    // warp-level for segments <= 4096, the rest block-level below
+    for (int b = wid; b < nbig; b += kWarps) {
+      int lp = sh.big_list[b];
+      int n = sm.p_cnt[lp];
+      if (n > 4096) continue;
+      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, lane, 32, [] { __syncwarp(); });
+    }
+    __syncthreads();
+    for (int b = 0; b < nbig; ++b) {
+      int lp = sh.big_list[b];
+      int n = sm.p_cnt[lp];
+      if (n <= 4096) continue;
+      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
+    }
+  } else {
+    // too many large segments for the list: one warp per segment, scanning all
+    for (int lp = wid; lp < nP; lp += kWarps) {
+      int n = sm.p_cnt[lp];
+      if (n <= 16 || n > 4096) continue;
+      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, lane, 32, [] { __syncwarp(); });
+    }
+    __syncthreads();
+    for (int lp = 0; lp < nP; ++lp) {
+      int n = sm.p_cnt[lp];
+      if (n <= 4096) continue;
+      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
+    }
+  }
+  __syncthreads();
+}
+
+// count = sum of kept children, V = sum of their valences clamped to T
+// (oversize valences are clamped, they get their own batch).
+// Kept children are the prefix [0, p_keep) of each (sorted) segment, or -- when
+// unsorted -- the non-kKeyMax entries of [0, p_cnt).
+__device__ void count_outputs(const KParams& kp, const SmemPtrs& sm, ShState& sh, int nP, int E) {
+  long long v = 0;
+  for (int e = threadIdx.x; e < E; e += kThreads) {
+    int lp = sm.lpof[e];
+    if (e - sm.p_eo[lp] >= sm.p_cnt[lp]) continue;
+    unsigned long long k = sm.cand[e];
+    if (k == kKeyMax) continue;
+    long long d = (long long)(k >> 32);
+    v += d < kp.T ? d : kp.T;
+  }
+  long long V = block_reduce_sum<long long>(v, sh.wtmpll);
+  int c = 0;
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) c += sm.p_keep[lp];
+  int C = block_reduce_sum<int32_t>(c, sh.wtmp32);
+  if (threadIdx.x == 0) { sh.count = C; sh.V = V; }
+  __syncthreads();
+}
+
+// Output (Alg. 5 ln 24-27): children in segment order at
+// o[out_off ...]; the RCM permutation is written reversed in the same pass
+// (perm[N-1-pos] = o[pos]) and optionally its inverse.
+// Requires sorted segments (kept = prefix of each segment).
+__device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                             int nP, int E, int out_off) {
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm.p_out[lp] = sm.p_keep[lp];
+  __syncthreads();
+  block_scan_array<int32_t>(sm.p_out, nP, sh.wtmp32);
+  int32_t* o = kp.o + P.o_base;
+  int32_t* perm = kp.perm + P.perm_base;
+  const int last = P.mat_n - 1;
+  for (int e = threadIdx.x; e < E; e += kThreads) {
+    int lp = sm.lpof[e];
+    int j = e - sm.p_eo[lp];
+    if (j >= sm.p_keep[lp]) continue;
+    int pos = out_off + sm.p_out[lp] + j;
+    int v = (int)(uint32_t)sm.cand[e];
+    o[pos] = v;
+    perm[last - pos] = v;
+    if (kp.iperm) kp.iperm[P.node_base + v] = last - pos;
+  }
+  __syncthreads();
+}
+
+// Unsorted variant (F_NO_SORT): kept = non-kKeyMax entries of each segment;
+// compact by a flat scan (order within a parent = discovery order).
+__device__ void compact_segments(const SmemPtrs& sm, ShState& sh, int nP) {
+  // per segment, move kept keys to the front (one thread per segment; debug path)
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
+    unsigned long long* a = sm.cand + sm.p_eo[lp];
+    int w = 0;
+    for (int i = 0; i < sm.p_cnt[lp]; ++i)
+      if (a[i] != kKeyMax) a[w++] = a[i];
+    for (int i = w; i < sm.p_cnt[lp]; ++i) a[i] = kKeyMax;
+  }
+  __syncthreads();
+}
+
+// ------------------------------------------------------ batch generation
+// Greedy cut of the ordered output (after an incoming overhang) into batches of
+// at most B_s nodes and at most T summed (clamped) valence; a node whose
+// valence reaches T gets a single-node batch.  `nb` slots were
+// reserved at q_off by signalCount (early generation); unused ones
+// are published as empty batches and skipped by the `next` link of
+// the last real batch.
+struct GenState {
+  int start;       // matrix-local position where the open batch starts
+  int cnt;         // nodes in the open batch
+  long long val;   // clamped valence sum of the open batch
+  int emitted;     // batches written so far
+  int pend_b, pend_e;  // last closed batch, not yet written (its `next` is unknown)
+  int has_pend;
+};
+
+__device__ __forceinline__ void publish_desc(Desc* d, int b, int e, int next, uint32_t epoch) {
+  d->o_begin = b;
+  d->o_end = e;
+  d->next = next;
+  __threadfence();
+  st_release_u32(&d->tag, epoch);
+}
+
+__device__ __forceinline__ void gen_close(const KParams& kp, GenState& g, int end, int q_off,
+                                          int nb, uint32_t epoch) {
+  if (g.has_pend) {
+    if (g.emitted < nb)   // never exceeded; guarded anyway
+      publish_desc(kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + g.emitted + 1, epoch);
+    else
+      latch_error(kp.ctl, ST_CAPACITY);
+    ++g.emitted;
+  }
+  g.pend_b = g.start;
+  g.pend_e = end;
+  g.has_pend = 1;
+  g.start = end;
+  g.cnt = 0;
+  g.val = 0;
+}
+
+// Consume one chunk of ordered nodes.  pre[i] (i <= m) = exclusive prefix over
+// the chunk's slots of (count << 40 | clamped valence); slot i's node sits at
+// matrix-local position base + (pre[i] >> 40).  Thread 0 only.
+__device__ void gen_chunk(const KParams& kp, GenState& g, const unsigned long long* pre, int m,
+                          int base, int q_off, int nb, uint32_t epoch) {
+  const unsigned long long kMaskV = (1ull << 40) - 1;
+  int a = 0;   // first slot not yet assigned
+  while (true) {
+    unsigned long long pa = pre[a];
+    unsigned long long pm = pre[m];
+    int ca = (int)(pa >> 40), cm = (int)(pm >> 40);
+    if (cm == ca) return;   // chunk exhausted
+    // largest slot s in (a, m] with cnt + (c(s)-c(a)) <= BS and val + (v(s)-v(a)) <= T
+    int lo = a, hi = m;
+    while (lo < hi) {
+      int mid = (lo + hi + 1) >> 1;
+      unsigned long long p = pre[mid];
+      int c = (int)(p >> 40) - ca;
+      long long v = (long long)((p & kMaskV) - (pa & kMaskV));
+      if (g.cnt + c <= kp.BS && g.val + v <= kp.T) lo = mid; else hi = mid - 1;
+    }
+    int taken = (int)(pre[lo] >> 40) - ca;
+    if (taken == 0) {
+      // the next node does not fit the open batch: close it (never empty here
+      // because a single node always fits an empty batch: clamped valence <= T)
+      gen_close(kp, g, base + ca, q_off, nb, epoch);
+      continue;
+    }
+    g.cnt += taken;
+    g.val += (long long)((pre[lo] & kMaskV) - (pa & kMaskV));
+    a = lo;
+    // advance a past holes (slots contributing nothing)
+    if ((int)(pre[lo] >> 40) == cm) return;
+    gen_close(kp, g, base + (int)(pre[lo] >> 40), q_off, nb, epoch);
+  }
+}
+
+__device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, int nb,
+                           uint32_t epoch) {
+  if (g.cnt > 0) gen_close(kp, g, end, q_off, nb, epoch);
+  if (g.has_pend) {
+    if (g.emitted < nb) publish_desc(kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + nb, epoch);
+    else latch_error(kp.ctl, ST_CAPACITY);
+    ++g.emitted;
+    g.has_pend = 0;
+  }
+}
+
+// Build pre[] over this batch's slots in cand[] (after write_output), in place.
+__device__ void build_prefix(const KParams& kp, const SmemPtrs& sm, ShState& sh, int E) {
+  // each thread: contiguous chunk of slots; kept = j < p_keep[lp] (sorted segments)
+  const int per = (E + kThreads - 1) / kThreads;
+  const int b = threadIdx.x * per, e = min(E, b + per);
+  unsigned long long s = 0;
+  for (int i = b; i < e; ++i) {
+    int lp = sm.lpof[i];
+    if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
+      unsigned long long d = sm.cand[i] >> 32;
+      s += (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+    }
+  }
+  unsigned long long tot;
+  unsigned long long run = block_exclusive_scan<unsigned long long>(s, sh.wtmp64, tot);
+  for (int i = b; i < e; ++i) {
+    int lp = sm.lpof[i];
+    unsigned long long x = 0;
+    if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
+      unsigned long long d = sm.cand[i] >> 32;
+      x = (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+    }
+    sm.cand[i] = run;
+    run += x;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) sm.cand[E] = tot;
+  __syncthreads();
+}
+
+// Publish empty batches q_off + [from, nb) (all threads of warp 0).
+__device__ void publish_empties(const KParams& kp, int q_off, int from, int nb, uint32_t epoch) {
+  if (threadIdx.x < 32) {
+    for (int i = from + threadIdx.x; i < nb; i += 32) publish_desc(kp.desc + q_off + i, 0, 0, q_off + i + 1, epoch);
+  }
+}
+
+}  // namespace rcm

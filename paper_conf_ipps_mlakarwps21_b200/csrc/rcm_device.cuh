@@ -1,0 +1,200 @@
+// rcm_device.cuh -- device-side data structures and primitives of the batch-RCM
+// library (sm_100a).  Citations P:L<n> = /root/reference/PAPER.md line n.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace rcm {
+
+constexpr int kThreads = 512;               // threads per persistent worker block
+constexpr int kWarps = kThreads / 32;
+constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
+constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner
+constexpr uint64_t kKeyMax = ~0ull;         // removed / padding sort key
+
+// Signal states a batch receives from its predecessor (Alg. 5).
+enum : uint32_t { S_NONE = 0, S_DISCOVERED = 1, S_COUNTED = 2, S_COMPLETED = 3 };
+
+// Status codes (mirror rcm_status_t)
+enum : int32_t { ST_OK = 0, ST_BAD_CSR = 2, ST_NOT_SYM = 3, ST_CAPACITY = 5, ST_HANG = 6 };
+
+// Batch descriptor: a contiguous range [o_begin, o_end) of matrix-local output
+// positions.  `next` is the queue index of the chain successor
+// (skip-link over trailing empty batches).  `tag` = chain epoch,
+// written last with release semantics: tag == epoch <=> published.
+struct __align__(16) Desc {
+  int32_t o_begin, o_end, next;
+  uint32_t tag;
+};
+
+// Signal a batch receives from its chain predecessor:
+// word = epoch << 32 | state; payload valid once state >= S_COUNTED.
+struct __align__(16) Sig {
+  unsigned long long word;
+  int32_t out_off;    // matrix-local output position of this batch's first child
+  int32_t q_off;      // queue index where this batch's generated batches go
+  int32_t ovh_nodes;  // overhang forwarded to this batch
+  int32_t ovh_temp;   //   ... and its (clamped) valence sum
+  int32_t pad[2];
+};
+
+// One independent unit of work: a connected component of one matrix.
+struct Problem {
+  int64_t node_base;  // word[] index of local node 0
+  int64_t rp_base;    // row_ptr index of local node 0
+  int64_t ci_base;    // added to row_ptr values to index col_idx
+  int64_t o_base;     // o[] index of matrix-local position 0
+  int64_t perm_base;  // perm[] index of matrix-local position 0
+  int32_t mat_n;      // matrix size (perm[perm_base + mat_n-1-pos] = o[pos])
+  int32_t pos0;       // first matrix-local position of this problem
+  int32_t size;       // nodes to order (component size, or mat_n when unknown)
+  int32_t seed;       // local id of the seed
+  int32_t flags;      // bit0: may contain several components (solo restart allowed)
+  int32_t pad;
+};
+
+// Device control block (one per plan, persistent across launches).
+struct Ctl {
+  unsigned long long minkey;   // prologue: min (deg << 32 | id)
+  int32_t maxdeg;
+  int32_t status;              // latched error (0 = ok)
+  int32_t head;                // chain dequeue counter
+  int32_t done;                // chain early-termination flag
+  int32_t chain_total;         // nodes ordered after the chain-first pass
+  uint32_t epoch;              // chain epoch counter (descriptor / signal tags)
+  int32_t gbar_count;          // grid barrier
+  int32_t gbar_gen;
+  int32_t solo_next;           // solo problem dequeue counter
+  int32_t n_chain;             // number of chain problems in the list
+  int32_t n_solo;              // number of solo problems in the list
+  int32_t n_comp;              // number of components found (CC pass)
+  int32_t spill_cursor;        // oversize scratch allocation cursor
+  int32_t chain_cur;           // chain index currently processed
+  int32_t incomplete;          // 1 if the chain-first pass did not order every node
+  int32_t pad[15];
+};
+
+struct Stats {
+  unsigned long long generated, dequeued, executed, empty, redisc_early, redisc_late,
+      cand_spec, cand_removed, oversize, components, ovh_forwards, solo_problems;
+};
+
+// ----------------------------------------------------------------- memory ops
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int32_t ld_acquire_s32(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int32_t ld_relaxed_s32(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_s32(int32_t* p, int32_t v) {
+  asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_s32(int32_t* p, int32_t v) {
+  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+// L2-coherent load for data written by other blocks during this launch.
+__device__ __forceinline__ int32_t ld_cg_s32(const int32_t* p) { return __ldcg(p); }
+
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Spin-wait budget before the watchdog latches RCM_ERR_HANG (ns).
+constexpr uint64_t kWatchdogNs = 20ull * 1000 * 1000 * 1000;
+
+// --------------------------------------------------------------- block scan
+// Exclusive block-wide prefix sum of one value per thread (kThreads threads).
+// `warp_tmp` must hold kWarps + 1 elements of T in shared memory.
+template <typename T>
+__device__ __forceinline__ T block_exclusive_scan(T v, T* warp_tmp, T& total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  T x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T y = __shfl_up_sync(0xffffffffu, x, d);
+    if (lane >= d) x += y;
+  }
+  if (lane == 31) warp_tmp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    T w = (lane < kWarps) ? warp_tmp[lane] : T(0);
+    T s = w;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      T y = __shfl_up_sync(0xffffffffu, s, d);
+      if (lane >= d) s += y;
+    }
+    if (lane < kWarps) warp_tmp[lane] = s - w;
+    if (lane == kWarps - 1) warp_tmp[kWarps] = s;
+  }
+  __syncthreads();
+  T res = warp_tmp[wid] + x - v;
+  total = warp_tmp[kWarps];
+  __syncthreads();
+  return res;
+}
+
+template <typename T>
+__device__ __forceinline__ T block_reduce_sum(T v, T* warp_tmp) {
+  T tot;
+  block_exclusive_scan<T>(v, warp_tmp, tot);
+  return tot;
+}
+
+// Exclusive scan, in place, of a[0..len) in shared memory; returns the total.
+// Each thread scans a contiguous chunk (few block barriers).
+template <typename T>
+__device__ __forceinline__ T block_scan_array(T* a, int len, T* warp_tmp) {
+  const int per = (len + kThreads - 1) / kThreads;
+  const int b = threadIdx.x * per;
+  const int e = min(len, b + per);
+  T s = 0;
+  for (int i = b; i < e; ++i) s += a[i];
+  T tot;
+  T run = block_exclusive_scan<T>(s, warp_tmp, tot);
+  for (int i = b; i < e; ++i) {
+    T x = a[i];
+    a[i] = run;
+    run += x;
+  }
+  __syncthreads();
+  return tot;
+}
+
+__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) {
+    unsigned long long o = __shfl_xor_sync(0xffffffffu, v, d);
+    v = o < v ? o : v;
+  }
+  return v;
+}
+
+}  // namespace rcm

@@ -1,0 +1,178 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the serial oracle, element by
+element (bit-exact: the output is an integer permutation).  Run with -m gpu."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from verifier import verify
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def rcm():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_mlakarwps21_b200 as m
+    return m
+
+
+def _dev(g):
+    return (torch.from_numpy(np.ascontiguousarray(g.row_ptr)).cuda(),
+            torch.from_numpy(np.ascontiguousarray(g.col_idx)).cuda())
+
+
+def _run(rcm, g, mode, start, plan=None, **opts):
+    own = plan is None
+    if own:
+        plan = rcm.Plan(max(g.n, 1), max(g.nnz, 1), **opts)
+    rp, ci = _dev(g)
+    iperm = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    perm = plan.reorder(rp, ci, mode, start, iperm=iperm).cpu().numpy()
+    ip = iperm.cpu().numpy()
+    assert np.array_equal(ip[perm], np.arange(g.n))
+    stats = plan.stats()
+    if own:
+        plan.close()
+    return perm, stats
+
+
+def _tiny_graphs():
+    gs = [synth.path(1), synth.path(2), synth.path(7), synth.cycle(9), synth.star(12), synth.complete(9),
+          synth.binary_tree(63), synth.grid2d(7, 5), synth.grid2d(13, 40, True)]
+    gs += [synth.gnp(80, 0.05, s) for s in range(6)]
+    gs += [synth.gnp(60, 0.3, 50 + s, diag=True) for s in range(2)]
+    gs.append(synth.relabel(synth.grid3d_27(7, 6, 5), synth.randperm(210, 3)))
+    gs.append(synth.disjoint_union([synth.path(4), synth.star(30), synth.complete(5), synth.path(1),
+                                    synth.grid2d(9, 9)]))
+    return gs
+
+
+MODES = [(oracle.FIXED, "mid"), (oracle.MIN_DEGREE, None)]
+PATHS = {
+    "solo": dict(),
+    "chain": dict(flags=8, solo_threshold=-1),
+    "chain_bs1": dict(flags=8, solo_threshold=-1, batch_nodes=1),
+    "chain_bs3_noovh": dict(flags=8 | 1, solo_threshold=-1, batch_nodes=3),
+    "chain_noearly": dict(flags=8 | 2, solo_threshold=-1, batch_nodes=7, temp_elems=2304),
+}
+
+
+@pytest.mark.parametrize("path", list(PATHS))
+def test_tiny_families(rcm, path):
+    for g in _tiny_graphs():
+        for mode, s in MODES:
+            start = g.n // 2 if s == "mid" else 0
+            ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+            got, _ = _run(rcm, g, mode, start, **PATHS[path])
+            assert np.array_equal(got, ref), (path, g.n, mode)
+
+
+@pytest.mark.parametrize("cfg", [1, 2, 3, 4])
+@pytest.mark.parametrize("path", ["solo", "chain", "chain_bs3_noovh"])
+def test_config_small_twins(rcm, cfg, path):
+    g, mode, start = synth.config_graph(cfg, "small")
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    opts = dict(PATHS[path])
+    if path == "solo":
+        opts["solo_threshold"] = g.n
+    got, st = _run(rcm, g, mode, start, **opts, collect_stats=1)
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("opts", [
+    dict(batch_nodes=1), dict(batch_nodes=2), dict(batch_nodes=3), dict(batch_nodes=64),
+    dict(batch_nodes=1024), dict(temp_elems=2304), dict(blocks_per_sm=1), dict(flags=1), dict(flags=2),
+    dict(flags=3, batch_nodes=16, temp_elems=2304),
+])
+def test_sweep_invariance(rcm, opts):
+    g, mode, start = synth.config_graph(2, "small")
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    o = dict(solo_threshold=-1)
+    o.update(opts)
+    got, _ = _run(rcm, g, mode, start, **o)
+    assert np.array_equal(got, ref), opts
+
+
+def test_repeat_determinism_and_stats(rcm):
+    g, mode, start = synth.config_graph(2, "small")
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    plan = rcm.Plan(g.n, g.nnz, solo_threshold=-1, collect_stats=1, batch_nodes=64)
+    rp, ci = _dev(g)
+    for _ in range(30):
+        perm = plan.reorder(rp, ci, mode, start).cpu().numpy()
+        assert np.array_equal(perm, ref)
+        st = plan.stats()
+        # Fig. 3 semantics: generated >= dequeued >= executed
+        assert st["batches_generated"] + 1 >= st["batches_dequeued"] >= st["batches_executed"]
+        assert st["batches_executed"] + st["batches_empty"] <= st["batches_dequeued"]
+        assert st["components"] == 1
+    plan.close()
+
+
+@pytest.mark.parametrize("cfg", [1, 2])
+def test_full_config_parity(rcm, cfg):
+    g, mode, start = synth.config_graph(cfg)
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    got, st = _run(rcm, g, mode, start, collect_stats=1)
+    assert np.array_equal(got, ref)
+    assert verify(g.row_ptr, g.col_idx, got, mode, start) is None
+
+
+@pytest.mark.parametrize("cfg", [3, 4])
+def test_full_config_parity_disconnected(rcm, cfg):
+    g, mode, start = synth.config_graph(cfg)
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    got, st = _run(rcm, g, mode, start, collect_stats=1)
+    assert np.array_equal(got, ref)
+
+
+def test_gl_finder(rcm):
+    for g, r in [(synth.path(30), 0), (synth.grid2d(7, 5), 0), (synth.grid2d(40, 13), 0)]:
+        plan = rcm.Plan(g.n, g.nnz)
+        rp, ci = _dev(g)
+        assert plan.find_pseudo_peripheral(rp, ci, r) == oracle.gl(g.row_ptr, g.col_idx, r)
+        plan.close()
+    g, _, _ = synth.config_graph(2, "small")
+    plan = rcm.Plan(g.n, g.nnz, solo_threshold=-1)
+    rp, ci = _dev(g)
+    for r in [0, 17, 4000]:
+        assert plan.find_pseudo_peripheral(rp, ci, r) == oracle.gl(g.row_ptr, g.col_idx, r)
+    perm = plan.reorder(rp, ci, oracle.PSEUDO_PERIPHERAL, 0).cpu().numpy()
+    assert np.array_equal(perm, oracle.rcm(g.row_ptr, g.col_idx, oracle.PSEUDO_PERIPHERAL, 0))
+    plan.close()
+
+
+def test_batched_small(rcm):
+    b = synth.c5_batch(num=40, seed=5, lo=50, hi=3000)
+    ref = oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, oracle.MIN_DEGREE)
+    total, nnz = int(b.node_off[-1]), int(b.nnz_off[-1])
+    plan = rcm.Plan(total, nnz)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()  # noqa: E731
+    perm = plan.reorder_batched(t(b.node_off), t(b.nnz_off), t(b.row_ptr_local), t(b.col_idx_local),
+                                total, nnz).cpu().numpy()
+    assert np.array_equal(perm, ref)
+    # FIXED starts
+    starts = (np.arange(40) * 7919) % np.diff(b.node_off)
+    ref2 = oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, oracle.FIXED, starts)
+    perm2 = plan.reorder_batched(t(b.node_off), t(b.nnz_off), t(b.row_ptr_local), t(b.col_idx_local),
+                                 total, nnz, mode=oracle.FIXED, starts=t(starts.astype(np.int32))).cpu().numpy()
+    assert np.array_equal(perm2, ref2)
+    plan.close()
+
+
+def test_host_argument_errors(rcm):
+    g = synth.path(5)
+    plan = rcm.Plan(5, 8)
+    rp, ci = _dev(g)
+    perm = torch.empty(5, dtype=torch.int32, device="cuda")
+    with pytest.raises(rcm.RCMError):
+        rcm.rcm_reorder(plan.handle, 5, 8, rp, ci, oracle.FIXED, 7, perm)      # start out of range
+    with pytest.raises(rcm.RCMError):
+        rcm.rcm_reorder(plan.handle, 6, 8, rp, ci, oracle.FIXED, 0, perm)      # n above plan
+    plan.close()
