@@ -1,0 +1,319 @@
+#!/usr/bin/env python
+"""Benchmark of the batch-RCM hot path (one JSON line on rank 0).
+
+Workload (default, BASELINE.json configs[1]): C2 = 3D 27-point FEM-like grid
+100^3 (1,000,000 nodes, 26,463,592 nnz), diagonal stored, random relabel
+(seed 2), MIN_DEGREE start -- see DESIGN.md "Input recipe".  A step = one
+rcm_reorder call (prologue + traversal + fused reverse) on device-resident
+input; the L2 is flushed before every timed step (input ~110 MB < 126 MB L2).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--config 2|5]
+
+N > 1 (torchrun): C1-C4 are one connected graph each and stay on one GPU, so
+every rank reorders its own replica ("replicas only"); config 5
+shards independent matrices across ranks and gathers the permutations with
+NCCL.  --impl reference times the serial oracle (the deliberately slow
+baseline) on the host cores of rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+HBM_FALLBACK_GBS = 6650.0
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return HBM_FALLBACK_GBS, "fallback"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.f = None
+
+    def start(self):
+        try:
+            self.f = tempfile.NamedTemporaryFile("w+", delete=False, suffix=".csv")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.flush()
+        rows = [l.strip().split(",") for l in open(self.f.name) if l.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx.append(float(r[1]))
+                for nm, v in zip(names, r[2:6]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except Exception:
+                continue
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------- inputs
+def load_workload(cfg: int):
+    import synth
+    if cfg in (1, 2, 3, 4):
+        g, mode, start = synth.config_graph(cfg)
+        names = {1: "C1 2D 5-point Laplacian 64x64, shuffled labels, FIXED start 0",
+                 2: "C2 3D 27-point FEM-like grid 100^3, random relabel, MIN_DEGREE start",
+                 3: "C3 random geometric graph 4M nodes, mean degree 14, MIN_DEGREE start",
+                 4: "C4 R-MAT 2^22 (0.57,0.19,0.19,0.05) x 8 edge samples, MIN_DEGREE start"}
+        return g, mode, start, names[cfg]
+    raise ValueError(cfg)
+
+
+def traffic_from_profile(cfg: int):
+    p = os.path.join(ROOT, "profiles", f"traffic_c{cfg}.json")
+    if os.path.exists(p):
+        try:
+            return json.load(open(p)).get("dram_bytes_per_launch")
+        except Exception:
+            return None
+    return None
+
+
+# ------------------------------------------------------------ reference arm
+def run_reference(args, rank: int):
+    if rank != 0:
+        return
+    import oracle
+    g, mode, start, name = load_workload(args.config)
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+        ts.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(ts) / len(ts)
+    val = g.n / (ms * 1e-3) / 1e6
+    line = {
+        "impl": "reference", "metric": "RCM Mnodes/s (serial oracle, host)", "value": round(val, 3),
+        "unit": "Mnodes/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": "i32", "data": "synthetic",
+        "config": {"workload": name, "n": g.n, "nnz": g.nnz},
+        "cpu_baseline": {"value": round(val, 3), "unit": "Mnodes/s", "cores": 1, "kind": "oracle",
+                         "sample": f"full workload graph, {args.steps} timed runs of the serial oracle"},
+        "e2e": {"value": round(val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------- our arm
+def run_ours(args, rank: int, world: int, local_rank: int):
+    import torch
+    import paper_conf_ipps_mlakarwps21_b200 as rcm
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    g, mode, start, name = load_workload(args.config)
+    n, nnz = g.n, g.nnz
+    rp_h = torch.from_numpy(g.row_ptr).pin_memory()
+    ci_h = torch.from_numpy(g.col_idx).pin_memory()
+    rp = rp_h.to(dev)
+    ci = ci_h.to(dev)
+    perm = torch.empty(n, dtype=torch.int32, device=dev)
+    plan = rcm.Plan(n, nnz, collect_stats=0)
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
+
+    def step():
+        rcm.rcm_reorder(plan.handle, n, nnz, rp, ci, mode, start, perm)
+
+    for _ in range(args.warmup):
+        step()
+    st = rcm.rcm_sync_status(plan.handle)
+    if st != 0:
+        raise RuntimeError(f"rcm_reorder failed: {rcm.STATUS.get(st)}")
+
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local_rank) if rank == 0 else None
+    if sampler:
+        sampler.start()
+    evs = []
+    for _ in range(args.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        step()
+        e1.record(stream)
+        evs.append((e0, e1))
+    torch.cuda.synchronize()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    dev_ms = sum(step_ms)
+    if dist is not None:
+        t = torch.tensor([dev_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.barrier()
+        dev_ms = float(t.item())
+    clocks = sampler.stop() if sampler else None
+    st = rcm.rcm_sync_status(plan.handle)
+    if st != 0:
+        raise RuntimeError(f"rcm_reorder failed: {rcm.STATUS.get(st)}")
+    phases = plan.timing()
+
+    # one stats run (counters off in the timed loop)
+    splan = rcm.Plan(n, nnz, collect_stats=1)
+    splan.reorder(rp, ci, mode, start)
+    stats = splan.stats()
+    info = splan.info()
+    splan.close()
+
+    # e2e through the public API: pinned host CSR in, permutation out, per step
+    perm_h = torch.empty(n, dtype=torch.int32).pin_memory()
+    e2e_evs = []
+    if dist is not None:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for _ in range(args.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        rp.copy_(rp_h, non_blocking=True)
+        ci.copy_(ci_h, non_blocking=True)
+        step()
+        perm_h.copy_(perm, non_blocking=True)
+        e1.record(stream)
+        e2e_evs.append((e0, e1))
+    torch.cuda.synchronize()
+    e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_evs)
+    if dist is not None:
+        t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+
+    if rank != 0:
+        plan.close()
+        return
+    # parity of the benchmarked output against the oracle (and the CPU baseline)
+    import oracle
+    oracle.build()
+    ots = []
+    ref = None
+    for _ in range(3):
+        t0 = time.perf_counter()
+        ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+        ots.append(time.perf_counter() - t0)
+    o_ms = 1e3 * statistics.median(ots)
+    got = perm_h.numpy()
+    parity = bool(np.array_equal(got, ref))
+
+    ms = dev_ms / args.steps
+    value = world * n / (ms * 1e-3) / 1e6
+    e2e_val = world * n / (e2e_ms / args.steps * 1e-3) / 1e6
+    peak, peak_kind = _peaks()
+    csr_once = 4 * (n + 1) + 4 * nnz
+    alg_bytes = csr_once + 28 * n
+    kern_ms = statistics.mean(step_ms)           # the step is exactly one k_main launch
+    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
+    executed = max(1, stats["batches_executed"])
+    line = {
+        "metric": "RCM Mnodes/s (ms/matrix in config) vs host serial RCM; % of HBM roofline",
+        "value": round(value, 3), "unit": "Mnodes/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "i32", "data": "synthetic",
+        "config": {"workload": name, "n": n, "nnz": nnz, "ms_per_matrix": round(ms, 4),
+                   "l2": "flushed before every timed step (256 MB write)",
+                   "parallelism": "replicas only" if world > 1 else "single GPU",
+                   "parity_vs_oracle": "bit-identical" if parity else "MISMATCH",
+                   "plan": info},
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 3), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 6), "traffic": traffic_from_profile(args.config),
+                     "peak_kind": peak_kind, "kernel": "k_main",
+                     "algorithmic_bytes": alg_bytes,
+                     "csr_once_bytes": csr_once,
+                     "csr_once_frac": round(csr_once / (kern_ms * 1e-3) / 1e9 / peak, 6)},
+        "cpu_baseline": {"value": round(n / (o_ms * 1e-3) / 1e6, 3), "unit": "Mnodes/s", "cores": 1,
+                         "kind": "oracle", "ms": round(o_ms, 3),
+                         "sample": "full workload graph, serial oracle, median of 3 runs"},
+        "speedup_vs_oracle": round(o_ms / ms, 2),
+        "e2e": {"value": round(e2e_val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 4 * (n + 1) + 4 * nnz,
+                "d2h_bytes_per_step": 4 * n, "ms_per_step": round(e2e_ms / args.steps, 4)},
+        "gpu_launches": args.steps,
+        "clocks": clocks,
+        "phases_ms": {k: round(v, 4) for k, v in phases.items()},
+        "stats": stats,
+        "chain": {"ms_per_executed_batch": round(phases["traversal_ms"] / executed, 5)},
+    }
+    print(json.dumps(line), flush=True)
+    plan.close()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=2)
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local_rank = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        run_reference(args, rank)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -32,7 +32,7 @@ STATUS = {
 
 # every symbol include/rcm.h declares
 EXPORTS = ["rcm_default_options", "rcm_plan_create", "rcm_reorder", "rcm_reorder_batched",
-           "rcm_find_pseudo_peripheral", "rcm_sync_status", "rcm_get_stats", "rcm_plan_info",
+           "rcm_find_pseudo_peripheral", "rcm_sync_status", "rcm_get_stats", "rcm_get_timing", "rcm_plan_info",
            "rcm_plan_destroy", "rcm_status_string"]
 
 
@@ -80,12 +80,13 @@ def _load():
     lib.rcm_sync_status.argtypes = [vp, vp]
     lib.rcm_get_stats.argtypes = [vp, ctypes.POINTER(rcm_stats_t)]
     lib.rcm_plan_info.argtypes = [vp, ctypes.POINTER(ctypes.c_int64)]
+    lib.rcm_get_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_double)]
     lib.rcm_plan_destroy.argtypes = [vp]
     lib.rcm_plan_destroy.restype = None
     lib.rcm_status_string.argtypes = [i32]
     lib.rcm_status_string.restype = ctypes.c_char_p
     for f in ("rcm_plan_create", "rcm_reorder", "rcm_reorder_batched", "rcm_find_pseudo_peripheral",
-              "rcm_sync_status", "rcm_get_stats", "rcm_plan_info"):
+              "rcm_sync_status", "rcm_get_stats", "rcm_get_timing", "rcm_plan_info"):
         getattr(lib, f).restype = i32
     _lib = lib
     return lib
@@ -178,6 +179,13 @@ def rcm_get_stats(plan) -> dict:
     return s.as_dict()
 
 
+def rcm_get_timing(plan) -> dict:
+    a = (ctypes.c_double * 5)()
+    _check(_load().rcm_get_timing(plan, a), "rcm_get_timing")
+    return dict(zip(("prologue_ms", "setup_ms", "traversal_ms", "components_ms", "total_ms"),
+                    [float(x) for x in a]))
+
+
 def rcm_plan_info(plan) -> dict:
     a = (ctypes.c_int64 * 6)()
     _check(_load().rcm_plan_info(plan, a), "rcm_plan_info")
@@ -218,6 +226,9 @@ class Plan:
 
     def stats(self):
         return rcm_get_stats(self.handle)
+
+    def timing(self):
+        return rcm_get_timing(self.handle)
 
     def reorder(self, row_ptr, col_idx, mode=RCM_START_MIN_DEGREE, start=0, perm=None, iperm=None,
                 stream=None, sync=True):

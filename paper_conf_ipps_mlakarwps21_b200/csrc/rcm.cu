@@ -9,217 +9,240 @@
 #include <new>
 
 #include "../../include/rcm.h"
-#include "rcm_components.cuh"
 #include "rcm_workers.cuh"
+#include "rcm_components.cuh"
 
 using namespace rcm;
 
-// ===================================================================== kernels
+// ===================================================================== phases
 // a1 -- prologue: valence = row_ptr diff, owner word init, argmin of
 // (valence, id) (C-6 / MIN_DEGREE seed), max valence, optional CSR checks.
 // Four nodes per thread with an int4 row_ptr load and a one-element halo.
-__global__ void __launch_bounds__(256) k_prologue(const int32_t* __restrict__ row_ptr, int n,
-                                                  long long nnz, unsigned long long* __restrict__ word,
-                                                  Ctl* ctl, int validate, int vec) {
-  __shared__ unsigned long long smin[8];
-  __shared__ int smax[8];
-  __shared__ int sbad[8];
-  const int t = blockIdx.x * blockDim.x + threadIdx.x;
-  const int v0 = t * 4;
+__device__ void prologue_phase(const KParams& kp, const MainArgs& a, ShState& sh) {
+  const int n = a.n;
   unsigned long long best = kKeyMax;
   int mx = 0, bad = 0;
-  if (v0 < n) {
+  const int G = gthreads(kp);
+  for (int t = gtid(); t * 4 < n; t += G) {
+    const int v0 = t * 4;
     int r[5];
-    if (vec && v0 + 4 <= n) {
-      int4 q = __ldg(reinterpret_cast<const int4*>(row_ptr + v0));
+    if (a.vec && v0 + 4 <= n) {
+      int4 q = __ldg(reinterpret_cast<const int4*>(kp.row_ptr + v0));
       r[0] = q.x; r[1] = q.y; r[2] = q.z; r[3] = q.w;
-      r[4] = __ldg(row_ptr + v0 + 4);
+      r[4] = __ldg(kp.row_ptr + v0 + 4);
     } else {
-      for (int j = 0; j < 5; ++j) r[j] = (v0 + j <= n) ? __ldg(row_ptr + v0 + j) : 0;
+      for (int j = 0; j < 5; ++j) r[j] = (v0 + j <= n) ? __ldg(kp.row_ptr + v0 + j) : 0;
     }
     const int m = min(4, n - v0);
     unsigned long long w[4];
+#pragma unroll
     for (int j = 0; j < 4; ++j) {
       if (j < m) {
         int d = r[j + 1] - r[j];
         if (d < 0) { bad = 1; d = 0; }
         w[j] = ((unsigned long long)kInf << 32) | (uint32_t)d;
-        unsigned long long k = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)(v0 + j);
+        const unsigned long long k = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)(v0 + j);
         best = k < best ? k : best;
         mx = max(mx, d);
       }
     }
     if (m == 4) {
-      reinterpret_cast<ulonglong2*>(word + v0)[0] = make_ulonglong2(w[0], w[1]);
-      reinterpret_cast<ulonglong2*>(word + v0)[1] = make_ulonglong2(w[2], w[3]);
+      reinterpret_cast<ulonglong2*>(kp.word + v0)[0] = make_ulonglong2(w[0], w[1]);
+      reinterpret_cast<ulonglong2*>(kp.word + v0)[1] = make_ulonglong2(w[2], w[3]);
     } else {
-      for (int j = 0; j < m; ++j) word[v0 + j] = w[j];
+      for (int j = 0; j < m; ++j) kp.word[v0 + j] = w[j];
     }
-    if (validate) {
+    if (a.validate) {
       if (v0 == 0 && r[0] != 0) bad = 1;
-      if (v0 + m == n && (long long)r[m] != nnz) bad = 1;
+      if (v0 + m == n && (long long)r[m] != a.nnz) bad = 1;
+    }
+  }
+  if (a.validate >= 1) {   // every column index in range
+    for (long long i = gtid(); i < a.nnz; i += G) {
+      const int c = __ldg(kp.col_idx + i);
+      bad |= (c < 0 || c >= n);
     }
   }
   best = warp_min_u64(best);
   for (int d = 16; d > 0; d >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, d));
   bad = __any_sync(0xffffffffu, bad);
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if (lane == 0) { smin[wid] = best; smax[wid] = mx; sbad[wid] = bad; }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    for (int i = 1; i < (int)(blockDim.x >> 5); ++i) {
-      best = smin[i] < best ? smin[i] : best;
-      mx = max(mx, smax[i]);
-      bad |= sbad[i];
-    }
-    if (best != kKeyMax) atomicMin(&ctl->minkey, best);
-    if (mx) atomicMax(&ctl->maxdeg, mx);
-    if (bad) atomicCAS(&ctl->status, 0, ST_BAD_CSR);
+  if ((threadIdx.x & 31) == 0) {
+    if (best != kKeyMax) atomicMin(&kp.ctl->minkey, best);
+    if (mx) atomicMax(&kp.ctl->maxdeg, mx);
+    if (bad) atomicCAS(&kp.ctl->status, 0, ST_BAD_CSR);
   }
-}
-
-// validate >= 1: every column index in range.
-__global__ void k_validate_cols(const int32_t* __restrict__ col_idx, long long nnz, int n, Ctl* ctl) {
-  int bad = 0;
-  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < nnz;
-       i += (long long)gridDim.x * blockDim.x) {
-    int c = __ldg(col_idx + i);
-    bad |= (c < 0 || c >= n);
-  }
-  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicCAS(&ctl->status, 0, ST_BAD_CSR);
 }
 
 // validate == 2: structural symmetry -- for every (u, c) the row of c holds u.
-__global__ void k_validate_sym(const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
-                               int n, Ctl* ctl) {
+__device__ void validate_sym_phase(const KParams& kp, int n) {
   int bad = 0;
-  for (int u = blockIdx.x * blockDim.x + threadIdx.x; u < n; u += gridDim.x * blockDim.x) {
-    for (int e = row_ptr[u]; e < row_ptr[u + 1]; ++e) {
-      int c = col_idx[e];
+  for (int u = gtid(); u < n; u += gthreads(kp)) {
+    for (int e = __ldg(kp.row_ptr + u); e < __ldg(kp.row_ptr + u + 1); ++e) {
+      const int c = __ldg(kp.col_idx + e);
       if (c < 0 || c >= n) { bad = 1; continue; }
       bool found = false;
-      for (int f = row_ptr[c]; f < row_ptr[c + 1] && !found; ++f) found = col_idx[f] == u;
+      for (int f = __ldg(kp.row_ptr + c); f < __ldg(kp.row_ptr + c + 1) && !found; ++f)
+        found = __ldg(kp.col_idx + f) == u;
       bad |= !found;
     }
   }
-  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicCAS(&ctl->status, 0, ST_NOT_SYM);
+  if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicCAS(&kp.ctl->status, 0, ST_NOT_SYM);
 }
 
 // Batched prologue: per matrix k, local valences and the per-matrix argmin.
-__global__ void __launch_bounds__(256) k_prologue_batched(const int32_t* __restrict__ rp_local,
-                                                          const int64_t* __restrict__ node_off,
-                                                          int num, long long total,
-                                                          unsigned long long* __restrict__ word,
-                                                          unsigned long long* __restrict__ pm_key,
-                                                          Ctl* ctl) {
-  const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long base = (long long)blockIdx.x * blockDim.x; base < total; base += stride) {
+__device__ void prologue_batched_phase(const KParams& kp, const MainArgs& a) {
+  const long long stride = (long long)gthreads(kp);
+  for (long long base = (long long)blockIdx.x * kThreads; base < a.total; base += stride) {
     const long long g = base + threadIdx.x;   // warp-uniform loop; lanes past the end idle
-    const bool valid = g < total;
-    int k = 0;
+    const bool valid = g < a.total;
+    int k = -1;
     unsigned long long key = kKeyMax;
     if (valid) {
-      // matrix of g: largest k with node_off[k] <= g
-      int lo = 0, hi = num - 1;
+      int lo = 0, hi = a.num_mats - 1;         // matrix of g: largest k with node_off[k] <= g
       while (lo < hi) {
-        int mid = (lo + hi + 1) >> 1;
-        if (__ldg(node_off + mid) <= g) lo = mid; else hi = mid - 1;
+        const int mid = (lo + hi + 1) >> 1;
+        if (__ldg(a.node_off + mid) <= g) lo = mid; else hi = mid - 1;
       }
       k = lo;
-      const int v = (int)(g - __ldg(node_off + k));
-      const int d = max(__ldg(rp_local + g + k + 1) - __ldg(rp_local + g + k), 0);
-      word[g] = ((unsigned long long)kInf << 32) | (uint32_t)d;
+      const int v = (int)(g - __ldg(a.node_off + k));
+      const int d = max(__ldg(kp.row_ptr + g + k + 1) - __ldg(kp.row_ptr + g + k), 0);
+      kp.word[g] = ((unsigned long long)kInf << 32) | (uint32_t)d;
       key = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)v;
-    } else {
-      k = -1;
     }
-    // warp-aggregated min per matrix: lanes of one matrix are contiguous, so a
-    // segmented shuffle-down min leaves the segment minimum in its first lane
+    // lanes of one matrix are contiguous: a segmented shuffle-down min leaves
+    // the segment minimum in its first lane
     const unsigned peers = __match_any_sync(0xffffffffu, k);
     unsigned long long m = key;
     const int lane = threadIdx.x & 31;
     for (int off = 1; off < 32; off <<= 1) {
-      unsigned long long o2 = __shfl_down_sync(0xffffffffu, m, off);
-      int ko = __shfl_down_sync(0xffffffffu, k, off);
+      const unsigned long long o2 = __shfl_down_sync(0xffffffffu, m, off);
+      const int ko = __shfl_down_sync(0xffffffffu, k, off);
       if (lane + off < 32 && ko == k && o2 < m) m = o2;
     }
-    if (valid && (int)(threadIdx.x & 31) == __ffs(peers) - 1) atomicMin(pm_key + k, m);
+    if (valid && lane == __ffs(peers) - 1) atomicMin(a.pm_key + k, m);
   }
 }
 
-// Problem set-up for one graph: the chain-first pass (or one solo problem).
-__global__ void k_setup_single(Problem* chains, Problem* solos, Ctl* ctl, int n, int mode, int start,
-                               int solo, const int32_t* gl_seed) {
-  Problem P;
-  P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
-  P.mat_n = n; P.pos0 = 0; P.size = n;
-  P.seed = mode == RCM_START_FIXED ? start
-         : (gl_seed ? *gl_seed : (int)(uint32_t)ctl->minkey);
-  P.flags = solo ? 1 : 0;
-  P.pad = 0;
-  if (solo) { solos[0] = P; ctl->n_solo = 1; ctl->n_chain = 0; }
-  else { chains[0] = P; ctl->n_chain = 1; ctl->n_solo = 0; }
-  ctl->solo_next = 0;
-  ctl->spill_cursor = 0;
-  ctl->incomplete = 0;
-  ctl->chain_total = 0;
-  ctl->gbar_count = 0;
-}
-
-// Problem set-up for a batch of matrices: one solo problem per matrix (C5).
-__global__ void k_setup_batched(Problem* solos, Ctl* ctl, const int64_t* __restrict__ node_off,
-                                const int64_t* __restrict__ nnz_off, int num, int mode,
-                                const int32_t* __restrict__ starts,
-                                const unsigned long long* __restrict__ pm_key,
-                                const int32_t* __restrict__ order) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i == 0) {
-    ctl->n_solo = num; ctl->n_chain = 0; ctl->solo_next = 0; ctl->spill_cursor = 0;
-    ctl->incomplete = 0; ctl->chain_total = 0; ctl->gbar_count = 0;
-  }
-  if (i >= num) return;
-  const int k = order ? order[i] : i;
-  Problem P;
-  P.node_base = node_off[k];
-  P.rp_base = node_off[k] + k;
-  P.ci_base = nnz_off[k];
-  P.o_base = node_off[k];
-  P.perm_base = node_off[k];
-  P.mat_n = (int)(node_off[k + 1] - node_off[k]);
-  P.pos0 = 0;
-  P.size = P.mat_n;
-  P.seed = (mode == RCM_START_FIXED && starts) ? starts[k] : (int)(uint32_t)pm_key[k];
-  P.flags = 1;
-  P.pad = 0;
-  solos[i] = P;
-}
-
-// The persistent scheduler: every chain problem in turn on all blocks (grid
+// The scheduling phase: every chain problem in turn on all blocks (grid
 // barrier between chains), then the solo problems, one per block at a time.
-__global__ void __launch_bounds__(kThreads, 2) k_scheduler(KParams kp) {
-  extern __shared__ __align__(16) unsigned char dsm[];
-  __shared__ ShState sh;
-  SmemPtrs sm = carve_smem(dsm, kp.BS, kp.T);
-  const int nchain = ld_relaxed_s32(&kp.ctl->n_chain);
+__device__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
+  const int nchain = ld_cg_s32(&kp.ctl->n_chain);
   for (int c = 0; c < nchain; ++c) {
+    if (kp.chains[c].flags & 2) {   // PSEUDO_PERIPHERAL component: GL seed first (C-5)
+      const int x = gl_phase(kp, a.w, a.n, kp.chains[c].seed, sh);
+      if (blockIdx.x == 0 && threadIdx.x == 0) const_cast<Problem*>(kp.chains)[c].seed = x;
+      grid_barrier(kp);
+    }
     if (blockIdx.x == 0 && threadIdx.x == 0) chain_init(kp, kp.chains[c]);
     grid_barrier(kp);
-    if (ld_relaxed_s32(&kp.ctl->status)) return;
+    if (ld_cg_s32(&kp.ctl->status)) return;
     const uint32_t epoch = ld_acquire_u32(&kp.ctl->epoch);
     const Problem P = kp.chains[c];
     chain_worker(kp, P, sm, sh, epoch);
     grid_barrier(kp);
   }
-  const int nsolo = ld_relaxed_s32(&kp.ctl->n_solo);
+  const int nsolo = ld_cg_s32(&kp.ctl->n_solo);
   for (;;) {
     if (threadIdx.x == 0) sh.k = atomicAdd(&kp.ctl->solo_next, 1);
     __syncthreads();
     const int k = sh.k;
     __syncthreads();
-    if (k >= nsolo || ld_relaxed_s32(&kp.ctl->status)) break;
-    const Problem P = kp.solos[k];
-    if (P.size > 0) run_solo(kp, P, sm, sh);
+    if (k >= nsolo || ld_cg_s32(&kp.ctl->status)) break;
+    Problem P = kp.solos[k];
+    if (P.size > 0) run_solo(kp, P, sm, sh, a.w.lev);
   }
+}
+
+// One launch per call: reset -> prologue -> seed / problem set-up ->
+// traversal -> (components -> traversal).  Grid barriers between phases.
+__global__ void __launch_bounds__(kThreads, 2) k_main(KParams kp, MainArgs a) {
+  extern __shared__ __align__(16) unsigned char dsm[];
+  __shared__ ShState sh;
+  SmemPtrs sm = carve_smem(dsm, kp.BS, kp.T);
+  const int G = gthreads(kp);
+  // ---- phase 0: reset the per-call control state
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    Ctl* c = kp.ctl;
+    c->ts[0] = globaltimer();
+    c->minkey = kKeyMax; c->maxdeg = 0; c->status = 0; c->head = 0; c->done = 0; c->chain_total = 0;
+    c->solo_next = 0; c->n_chain = 0; c->n_solo = 0; c->n_comp = 0; c->spill_cursor = 0; c->incomplete = 0;
+    if (kp.collect_stats) *kp.stats = Stats{};
+  }
+  if (a.batched)
+    for (int k = gtid(); k < a.num_mats; k += G) a.pm_key[k] = kKeyMax;
+  if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.gl_only) {
+    const long long nn = a.batched ? a.total : a.n;
+    for (long long v = gtid(); v < nn; v += G) a.w.lev[v] = -1;
+  }
+  grid_barrier(kp);
+  // ---- phase 1: prologue (a1)
+  if (a.batched) prologue_batched_phase(kp, a);
+  else prologue_phase(kp, a, sh);
+  if (!a.batched && a.validate == 2) validate_sym_phase(kp, a.n);
+  grid_barrier(kp);
+  stamp(kp, 1);
+  if (ld_cg_s32(&kp.ctl->status)) return;
+  if (a.gl_only) {   // rcm_find_pseudo_peripheral
+    const int x = gl_phase(kp, a.w, a.n, a.gl_start, sh);
+    if (gtid() == 0) *a.gl_out = x;
+    stamp(kp, 4);
+    return;
+  }
+  // ---- phase 2: problems
+  const int gl_flag = a.mode == RCM_START_PSEUDO_PERIPHERAL ? 2 : 0;
+  if (a.batched) {
+    // LPT: largest matrices first (solo workers dequeue in this order)
+    for (int k = gtid(); k < a.num_mats; k += G) {
+      const long long sz = a.node_off[k + 1] - a.node_off[k];
+      a.w.keys0[k] = ((unsigned long long)(0xffffffffu - (uint32_t)sz) << 32) | (uint32_t)k;
+      a.w.vals0[k] = k;
+    }
+    if (gtid() == 0) { a.w.sctl[0] = a.num_mats; a.w.sctl[1] = 0; }
+    grid_barrier(kp);
+    radix_sort_phase(kp, a.w, 64, reinterpret_cast<int32_t*>(sm.cand), sh);
+    const int32_t* order = ld_cg_s32(a.w.sctl + 1) ? a.w.vals1 : a.w.vals0;
+    Problem* solos = const_cast<Problem*>(kp.solos);
+    for (int i = gtid(); i < a.num_mats; i += G) {
+      const int k = __ldcg(order + i);
+      Problem P;
+      P.node_base = a.node_off[k];
+      P.rp_base = a.node_off[k] + k;
+      P.ci_base = a.nnz_off[k];
+      P.o_base = a.node_off[k];
+      P.perm_base = a.node_off[k];
+      P.mat_n = (int)(a.node_off[k + 1] - a.node_off[k]);
+      P.pos0 = 0;
+      P.size = P.mat_n;
+      P.seed = (a.mode == RCM_START_FIXED && a.starts) ? a.starts[k] : (int)(uint32_t)__ldcg(a.pm_key + k);
+      P.flags = 1 | gl_flag;
+      P.pad = 0;
+      solos[i] = P;
+    }
+    if (gtid() == 0) kp.ctl->n_solo = a.num_mats;
+  } else {
+    int seed = a.mode == RCM_START_FIXED ? a.start : (int)(uint32_t)__ldcg(&kp.ctl->minkey);
+    if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.solo) seed = gl_phase(kp, a.w, a.n, seed, sh);
+    if (gtid() == 0) {
+      Problem P;
+      P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
+      P.mat_n = a.n; P.pos0 = 0; P.size = a.n; P.seed = seed; P.pad = 0;
+      if (a.solo) { P.flags = 1 | gl_flag; const_cast<Problem*>(kp.solos)[0] = P; kp.ctl->n_solo = 1; }
+      else { P.flags = 0; const_cast<Problem*>(kp.chains)[0] = P; kp.ctl->n_chain = 1; }
+    }
+  }
+  grid_barrier(kp);
+  stamp(kp, 2);
+  // ---- phase 3: the traversal (a2-a12)
+  schedule_phase(kp, a, sm, sh);
+  grid_barrier(kp);
+  stamp(kp, 3);
+  // ---- phase 4: components left over by the chain-first pass (a13)
+  if (!a.batched && !a.solo && ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
+    cc_phase(kp, a, sm, sh);
+    schedule_phase(kp, a, sm, sh);
+    grid_barrier(kp);
+  }
+  stamp(kp, 4);
 }
 
 // ======================================================================= host
@@ -239,18 +262,16 @@ struct rcm_plan {
   Problem* solos = nullptr;
   unsigned long long* pm_key = nullptr;
   unsigned long long* spill = nullptr;
-  CompWS comp{};
-  int32_t* gl_out = nullptr;
-  int32_t last_status = 0;
+  CompWS w{};
 };
 
 static rcm_status_t cuda_fail(cudaError_t e) {
   if (e == cudaErrorMemoryAllocation) return RCM_ERR_OUT_OF_MEMORY;
   return RCM_ERR_CUDA;
 }
-#define CK(x)                                   \
-  do {                                          \
-    cudaError_t _e = (x);                       \
+#define CK(x)                                    \
+  do {                                           \
+    cudaError_t _e = (x);                        \
     if (_e != cudaSuccess) return cuda_fail(_e); \
   } while (0)
 
@@ -273,12 +294,17 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
   return "unknown status";
 }
 
+static void free_all(rcm_plan* p) {
+  void* ptrs[] = {p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+                  p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
+                  p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
+                  p->w.gctl, p->w.gkey};
+  for (void* q : ptrs) cudaFree(q);
+}
+
 extern "C" void rcm_plan_destroy(rcm_plan_t p) {
   if (!p) return;
-  cudaFree(p->word); cudaFree(p->o); cudaFree(p->desc); cudaFree(p->sig); cudaFree(p->ctl);
-  cudaFree(p->stats); cudaFree(p->chains); cudaFree(p->solos); cudaFree(p->pm_key);
-  cudaFree(p->spill); cudaFree(p->gl_out);
-  comp_free(p->comp);
+  free_all(p);
   delete p;
 }
 
@@ -297,60 +323,63 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   }
   p->n_max = n_max;
   p->nnz_max = nnz_max;
-  cudaError_t e = cudaGetDevice(&p->device);
-  if (e != cudaSuccess) { delete p; return RCM_ERR_CUDA; }
+  if (cudaGetDevice(&p->device) != cudaSuccess) { delete p; return RCM_ERR_CUDA; }
   cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->device);
-  int smem_optin = 0;
+  int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
-  int smem_sm = 0;
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
   p->BS = o.batch_nodes ? o.batch_nodes : 512;
-  int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
+  const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
   const size_t static_sh = sizeof(ShState) + 64;
   // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per block)
-  size_t per_block = std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
+  const size_t per_block =
+      std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
   int T = o.temp_elems;
-  if (!T) {
-    size_t fixed = smem_bytes(p->BS, 0);
-    T = (int)((per_block - fixed) / 10);
-    T = T / 256 * 256;
-  }
+  if (!T) T = (int)((per_block - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
   if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;
   }
   p->T = T;
   p->smem = smem_bytes(p->BS, T);
-  e = cudaFuncSetAttribute(k_scheduler, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem);
-  if (e != cudaSuccess) { delete p; return RCM_ERR_CUDA; }
+  if (cudaFuncSetAttribute(k_main, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
+    delete p;
+    return RCM_ERR_CUDA;
+  }
   int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_scheduler, kThreads, p->smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_main, kThreads, p->smem);
   if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
-  p->nblocks = std::min(occ, bps) * p->num_sms;
+  p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
   // queue bound: sum over generating batches of floor(N/B) + max(1, ceil(2V/T))
-  int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
+  const int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
   p->qcap = o.queue_capacity ? o.queue_capacity : std::min<int64_t>(qb, (1ll << 31) - 2);
   p->prob_cap = std::max<int64_t>(1, n_max / 2 + 1);
   p->spill_cap = n_max;
+  const int64_t n = n_max;
+  const int64_t tiles = (n + kSortTile - 1) / kSortTile + 1;
   rcm_status_t st = RCM_OK;
-#define AL(ptr, bytes)                                                  \
-  do {                                                                  \
-    cudaError_t _e = cudaMalloc((void**)&(ptr), (bytes));               \
-    if (_e != cudaSuccess) { st = cuda_fail(_e); goto fail; }           \
+#define AL(ptr, bytes)                                        \
+  do {                                                        \
+    cudaError_t _e = cudaMalloc((void**)&(ptr), (bytes));     \
+    if (_e != cudaSuccess) { st = cuda_fail(_e); goto fail; } \
   } while (0)
-  AL(p->word, sizeof(unsigned long long) * n_max);
-  AL(p->o, sizeof(int32_t) * n_max);
+  AL(p->word, 8 * n);
+  AL(p->o, 4 * n);
   AL(p->desc, sizeof(Desc) * p->qcap);
   AL(p->sig, sizeof(Sig) * (p->qcap + 1));
   AL(p->ctl, sizeof(Ctl));
   AL(p->stats, sizeof(Stats));
   AL(p->chains, sizeof(Problem) * p->prob_cap);
   AL(p->solos, sizeof(Problem) * p->prob_cap);
-  AL(p->pm_key, sizeof(unsigned long long) * p->prob_cap);
-  AL(p->spill, sizeof(unsigned long long) * 2 * p->spill_cap);
-  AL(p->gl_out, sizeof(int32_t) * 4);
-  if (comp_alloc(p->comp, n_max) != cudaSuccess) { st = RCM_ERR_OUT_OF_MEMORY; goto fail; }
+  AL(p->pm_key, 8 * p->prob_cap);
+  AL(p->spill, 8 * 2 * p->spill_cap);
+  AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
+  AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
+  AL(p->w.offs, 8 * (n + 1)); AL(p->w.hist, 4 * 256 * tiles); AL(p->w.sctl, 4 * 64);
+  AL(p->w.order, 4 * n); AL(p->w.lev, 4 * n); AL(p->w.front0, 4 * n); AL(p->w.front1, 4 * n);
+  AL(p->w.gctl, 4 * 64); AL(p->w.gkey, 8 * 64);
 #undef AL
+  p->w.cap = n;
   // descriptors / signals start with tag 0 (epochs start at 1)
   if (cudaMemset(p->desc, 0, sizeof(Desc) * p->qcap) != cudaSuccess ||
       cudaMemset(p->sig, 0, sizeof(Sig) * (p->qcap + 1)) != cudaSuccess ||
@@ -392,26 +421,24 @@ static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* 
   return kp;
 }
 
-// Reset the per-call parts of the control block (keeps the epoch counter).
-__global__ void k_reset_ctl(Ctl* ctl, Stats* stats) {
-  ctl->minkey = kKeyMax;
-  ctl->maxdeg = 0;
-  ctl->status = 0;
-  ctl->head = 0;
-  ctl->done = 0;
-  ctl->chain_total = 0;
-  ctl->gbar_count = 0;
-  ctl->solo_next = 0;
-  ctl->n_chain = 0;
-  ctl->n_solo = 0;
-  ctl->n_comp = 0;
-  ctl->spill_cursor = 0;
-  ctl->incomplete = 0;
-  if (stats) *stats = Stats{};
+static MainArgs make_args(rcm_plan* p) {
+  MainArgs a;
+  std::memset(&a, 0, sizeof(a));
+  a.w = p->w;
+  a.prob_cap = p->prob_cap;
+  a.validate = p->opt.validate;
+  a.thr = p->opt.solo_threshold == 0 ? 4096 : p->opt.solo_threshold;
+  return a;
 }
 
-static rcm_status_t launch_scheduler(rcm_plan* p, const KParams& kp, cudaStream_t s) {
-  k_scheduler<<<p->nblocks, kThreads, p->smem, s>>>(kp);
+static int bits_for(int64_t x) {
+  int b = 0;
+  while (b < 62 && (1ll << b) <= x) ++b;
+  return b;
+}
+
+static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& a, cudaStream_t s) {
+  k_main<<<p->nblocks, kThreads, p->smem, s>>>(kp, a);
   CK(cudaGetLastError());
   return RCM_OK;
 }
@@ -423,37 +450,16 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   if (n > p->n_max || nnz > p->nnz_max || nnz >= (1ll << 31)) return RCM_ERR_INVALID_ARGUMENT;
   if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
   if (mode == RCM_START_FIXED && (start < 0 || start >= n)) return RCM_ERR_INVALID_ARGUMENT;
-  cudaStream_t s = (cudaStream_t)stream;
   KParams kp = make_kparams(p, row_ptr, col_idx, perm, iperm);
-  k_reset_ctl<<<1, 1, 0, s>>>(p->ctl, p->stats);
-  const int vec = ((reinterpret_cast<uintptr_t>(row_ptr) & 15) == 0) ? 1 : 0;
-  const int nthr4 = (n + 3) / 4;
-  k_prologue<<<(nthr4 + 255) / 256, 256, 0, s>>>(row_ptr, n, nnz, p->word, p->ctl, p->opt.validate, vec);
-  if (p->opt.validate >= 1 && nnz > 0)
-    k_validate_cols<<<std::min<long long>((nnz + 255) / 256, 4096), 256, 0, s>>>(col_idx, nnz, n, p->ctl);
-  if (p->opt.validate == 2)
-    k_validate_sym<<<std::min((n + 255) / 256, 4096), 256, 0, s>>>(row_ptr, col_idx, n, p->ctl);
-  const int32_t* gl_seed = nullptr;
-  if (mode == RCM_START_PSEUDO_PERIPHERAL) {
-    rcm_status_t st = gl_launch(p->comp, row_ptr, col_idx, n, p->word, p->ctl, nullptr, p->gl_out, s);
-    if (st != RCM_OK) return st;
-    gl_seed = p->gl_out;
-  }
-  const int thr = p->opt.solo_threshold == 0 ? 4096 : p->opt.solo_threshold;
-  const int solo = (!(p->opt.flags & RCM_FLAG_FORCE_CHAIN) && thr > 0 && n <= thr) ? 1 : 0;
-  k_setup_single<<<1, 1, 0, s>>>(p->chains, p->solos, p->ctl, n, (int)mode, start, solo, gl_seed);
-  CK(cudaGetLastError());
-  rcm_status_t st = launch_scheduler(p, kp, s);
-  if (st != RCM_OK) return st;
-  if (!solo) {
-    // a13: components left over by the chain-first pass (C-6).  All kernels of
-    // this stage exit immediately when the first pass ordered every node.
-    st = comp_stage(p->comp, kp, n, nnz, (int)mode, thr, p->prob_cap, s);
-    if (st != RCM_OK) return st;
-    st = launch_scheduler(p, kp, s);
-    if (st != RCM_OK) return st;
-  }
-  return RCM_OK;
+  MainArgs a = make_args(p);
+  a.n = n;
+  a.nnz = nnz;
+  a.mode = (int)mode;
+  a.start = start;
+  a.vec = ((reinterpret_cast<uintptr_t>(row_ptr) & 15) == 0) ? 1 : 0;
+  a.solo = (!(p->opt.flags & RCM_FLAG_FORCE_CHAIN) && a.thr > 0 && n <= a.thr) ? 1 : 0;
+  a.idbits = bits_for(n - 1 > 0 ? n - 1 : 1);
+  return launch_main(p, kp, a, (cudaStream_t)stream);
 }
 
 extern "C" rcm_status_t rcm_reorder_batched(rcm_plan_t p, int32_t num_mats, int64_t total_nodes,
@@ -467,29 +473,18 @@ extern "C" rcm_status_t rcm_reorder_batched(rcm_plan_t p, int32_t num_mats, int6
   if (total_nodes > p->n_max || total_nnz > p->nnz_max || num_mats > p->prob_cap) return RCM_ERR_INVALID_ARGUMENT;
   if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
   if (mode == RCM_START_FIXED && !starts) return RCM_ERR_INVALID_ARGUMENT;
-  cudaStream_t s = (cudaStream_t)stream;
   KParams kp = make_kparams(p, row_ptr_local, col_idx_local, perm_local, nullptr);
-  k_reset_ctl<<<1, 1, 0, s>>>(p->ctl, p->stats);
-  CK(cudaMemsetAsync(p->pm_key, 0xff, sizeof(unsigned long long) * num_mats, s));
-  const long long blocks = std::min<long long>((total_nodes + 255) / 256, 65535);
-  k_prologue_batched<<<(int)blocks, 256, 0, s>>>(row_ptr_local, node_off, num_mats, total_nodes, p->word,
-                                                 p->pm_key, p->ctl);
-  const int32_t* order = nullptr;
-  if (num_mats > 1) {
-    // LPT: largest matrices first (the solo workers dequeue in this order)
-    rcm_status_t st = comp_order_by_size(p->comp, node_off, num_mats, s);
-    if (st != RCM_OK) return st;
-    order = p->comp.order;
-  }
-  if (mode == RCM_START_PSEUDO_PERIPHERAL) {
-    rcm_status_t st = gl_batched(p->comp, row_ptr_local, col_idx_local, node_off, nnz_off, num_mats,
-                                 p->pm_key, s);
-    if (st != RCM_OK) return st;
-  }
-  k_setup_batched<<<(num_mats + 255) / 256, 256, 0, s>>>(p->solos, p->ctl, node_off, nnz_off, num_mats,
-                                                         (int)mode, starts, p->pm_key, order);
-  CK(cudaGetLastError());
-  return launch_scheduler(p, kp, s);
+  MainArgs a = make_args(p);
+  a.batched = 1;
+  a.mode = (int)mode;
+  a.num_mats = num_mats;
+  a.total = total_nodes;
+  a.nnz = total_nnz;
+  a.node_off = node_off;
+  a.nnz_off = nnz_off;
+  a.starts = starts;
+  a.pm_key = p->pm_key;
+  return launch_main(p, kp, a, (cudaStream_t)stream);
 }
 
 extern "C" rcm_status_t rcm_find_pseudo_peripheral(rcm_plan_t p, int32_t n, int64_t nnz,
@@ -498,11 +493,17 @@ extern "C" rcm_status_t rcm_find_pseudo_peripheral(rcm_plan_t p, int32_t n, int6
   if (!p || !row_ptr || !out || n <= 0 || start < 0 || start >= n || nnz < 0 || (nnz > 0 && !col_idx))
     return RCM_ERR_INVALID_ARGUMENT;
   if (n > p->n_max || nnz > p->nnz_max) return RCM_ERR_INVALID_ARGUMENT;
-  cudaStream_t s = (cudaStream_t)stream;
-  k_reset_ctl<<<1, 1, 0, s>>>(p->ctl, nullptr);
-  const int vec = ((reinterpret_cast<uintptr_t>(row_ptr) & 15) == 0) ? 1 : 0;
-  k_prologue<<<((n + 3) / 4 + 255) / 256, 256, 0, s>>>(row_ptr, n, nnz, p->word, p->ctl, 0, vec);
-  return gl_launch(p->comp, row_ptr, col_idx, n, p->word, p->ctl, &start, out, s);
+  KParams kp = make_kparams(p, row_ptr, col_idx, nullptr, nullptr);
+  MainArgs a = make_args(p);
+  a.n = n;
+  a.nnz = nnz;
+  a.mode = RCM_START_PSEUDO_PERIPHERAL;
+  a.vec = ((reinterpret_cast<uintptr_t>(row_ptr) & 15) == 0) ? 1 : 0;
+  a.gl_only = 1;
+  a.gl_start = start;
+  a.gl_out = out;
+  a.validate = 0;
+  return launch_main(p, kp, a, (cudaStream_t)stream);
 }
 
 extern "C" rcm_status_t rcm_sync_status(rcm_plan_t p, void* stream) {
@@ -510,7 +511,6 @@ extern "C" rcm_status_t rcm_sync_status(rcm_plan_t p, void* stream) {
   CK(cudaStreamSynchronize((cudaStream_t)stream));
   int32_t st = 0;
   CK(cudaMemcpy(&st, &p->ctl->status, sizeof(int32_t), cudaMemcpyDeviceToHost));
-  p->last_status = st;
   return (rcm_status_t)st;
 }
 
@@ -518,7 +518,7 @@ extern "C" rcm_status_t rcm_get_stats(rcm_plan_t p, rcm_stats_t* out) {
   if (!p || !out) return RCM_ERR_INVALID_ARGUMENT;
   Stats s;
   CK(cudaMemcpy(&s, p->stats, sizeof(Stats), cudaMemcpyDeviceToHost));
-  out->batches_generated = (int64_t)s.generated + 0;
+  out->batches_generated = (int64_t)s.generated;
   out->batches_dequeued = (int64_t)s.dequeued;
   out->batches_executed = (int64_t)s.executed;
   out->batches_empty = (int64_t)s.empty;
@@ -530,6 +530,20 @@ extern "C" rcm_status_t rcm_get_stats(rcm_plan_t p, rcm_stats_t* out) {
   out->components = (int64_t)s.components;
   out->overhang_forwards = (int64_t)s.ovh_forwards;
   out->solo_problems = (int64_t)s.solo_problems;
+  return RCM_OK;
+}
+
+extern "C" rcm_status_t rcm_get_timing(rcm_plan_t p, double* out_ms) {
+  if (!p || !out_ms) return RCM_ERR_INVALID_ARGUMENT;
+  unsigned long long ts[8];
+  CK(cudaMemcpy(ts, p->ctl->ts, sizeof(ts), cudaMemcpyDeviceToHost));
+  // [prologue, seed + set-up, traversal, components + their traversal, total]
+  auto d = [&](int a, int b) { return ts[b] >= ts[a] ? (double)(ts[b] - ts[a]) * 1e-6 : 0.0; };
+  out_ms[0] = d(0, 1);
+  out_ms[1] = d(1, 2);
+  out_ms[2] = d(2, 3);
+  out_ms[3] = d(3, 4);
+  out_ms[4] = d(0, 4);
   return RCM_OK;
 }
 

@@ -71,7 +71,8 @@ struct Ctl {
   int32_t spill_cursor;        // oversize scratch allocation cursor
   int32_t chain_cur;           // chain index currently processed
   int32_t incomplete;          // 1 if the chain-first pass did not order every node
-  int32_t pad[15];
+  int32_t pad[3];
+  unsigned long long ts[8];    // phase timestamps (%globaltimer ns) of the last call
 };
 
 struct Stats {

@@ -551,12 +551,76 @@ __device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs
 }
 
 // ------------------------------------------------------------- solo worker
+// Block-level BFS inside one component for the pseudo-peripheral finder
+// (P:L365-375): the queue lives in the component's still-unwritten output
+// range q[], levels in lev[] (-1 = unvisited; reset before returning).
+// Returns the number of levels; sh.minkey = min (valence, id) of the last level.
+__device__ int block_bfs(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
+  int32_t* lv = lev + P.node_base;
+  const int32_t* rp = kp.row_ptr + P.rp_base;
+  const int32_t* col = kp.col_idx + P.ci_base;
+  if (threadIdx.x == 0) { q[0] = r; lv[r] = 0; sh.written = 1; }
+  __syncthreads();
+  int head = 0, tail = 1, level = 0, lb = 0;
+  for (;;) {
+    for (int i = head + threadIdx.x; i < tail; i += kThreads) {
+      const int p = q[i];
+      for (int e = __ldg(rp + p); e < __ldg(rp + p + 1); ++e) {
+        const int c = __ldg(col + e);
+        if (ld_cg_s32(lv + c) < 0 && atomicCAS(lv + c, -1, level + 1) == -1) q[atomicAdd(&sh.written, 1)] = c;
+      }
+    }
+    __syncthreads();
+    const int nt = sh.written;
+    __syncthreads();
+    if (nt == tail) break;
+    lb = tail;
+    head = tail;
+    tail = nt;
+    ++level;
+  }
+  unsigned long long best = kKeyMax;
+  const unsigned long long* word = kp.word + P.node_base;
+  for (int i = lb + threadIdx.x; i < tail; i += kThreads) {
+    const int v = q[i];
+    const unsigned long long k = ((ld_relaxed_u64(word + v) & 0xffffffffull) << 32) | (uint32_t)v;
+    best = k < best ? k : best;
+  }
+  best = warp_min_u64(best);
+  if ((threadIdx.x & 31) == 0) sh.wtmp64[threadIdx.x >> 5] = best;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    unsigned long long b = threadIdx.x < kWarps ? sh.wtmp64[threadIdx.x] : kKeyMax;
+    b = warp_min_u64(b);
+    if (threadIdx.x == 0) sh.minkey = b;
+  }
+  for (int i = threadIdx.x; i < tail; i += kThreads) lv[q[i]] = -1;
+  __syncthreads();
+  return level + 1;
+}
+
+// GL finder (C-5) from r inside its component, block-level.
+__device__ int block_gl(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
+  int nl = block_bfs(kp, P, q, lev, r, sh);
+  int x = (int)(uint32_t)sh.minkey;
+  __syncthreads();
+  for (;;) {
+    const int nx = block_bfs(kp, P, q, lev, x, sh);
+    if (nx <= nl) return x;   // same level count: "use the last node"
+    nl = nx;
+    x = (int)(uint32_t)sh.minkey;
+    __syncthreads();
+  }
+}
+
 // One block orders a whole component (or a whole small matrix, restarting at
 // the C-6 seed when a component is exhausted) with the same batch steps but
 // without the signalling chain: batches are consecutive output ranges.
-__device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh) {
+__device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh, int32_t* lev) {
+  int seed = P.seed;
+  if (P.flags & 2) seed = block_gl(kp, P, kp.o + P.o_base + P.pos0, lev, seed, sh);
   if (threadIdx.x == 0) {
-    place_root(kp, P, P.seed, P.pos0);
+    place_root(kp, P, seed, P.pos0);
     stat_add(kp, &kp.stats->solo_problems, 1);
     stat_add(kp, &kp.stats->components, 1);
   }
@@ -575,6 +639,7 @@ __device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm
         if (threadIdx.x == 0) latch_error(kp.ctl, ST_BAD_CSR);
         break;
       }
+      if (P.flags & 2) s = block_gl(kp, P, kp.o + P.o_base + written, lev, s, sh);
       if (threadIdx.x == 0) {
         place_root(kp, P, s, written);
         stat_add(kp, &kp.stats->components, 1);
