@@ -23,6 +23,7 @@ RCM_FLAG_NO_OVERHANG = 0x1
 RCM_FLAG_NO_EARLY = 0x2
 RCM_FLAG_NO_SORT = 0x4
 RCM_FLAG_FORCE_CHAIN = 0x8
+RCM_FLAG_SERIAL_CHAIN = 0x10
 
 STATUS = {
     0: "RCM_OK", 1: "RCM_ERR_INVALID_ARGUMENT", 2: "RCM_ERR_BAD_CSR", 3: "RCM_ERR_NOT_SYMMETRIC",
@@ -180,9 +181,10 @@ def rcm_get_stats(plan) -> dict:
 
 
 def rcm_get_timing(plan) -> dict:
-    a = (ctypes.c_double * 5)()
+    a = (ctypes.c_double * 7)()
     _check(_load().rcm_get_timing(plan, a), "rcm_get_timing")
-    return dict(zip(("prologue_ms", "setup_ms", "traversal_ms", "components_ms", "total_ms"),
+    return dict(zip(("prologue_ms", "setup_ms", "traversal_ms", "components_ms", "total_ms",
+                     "cc_label_ms", "cc_sort_layout_ms"),
                     [float(x) for x in a]))
 
 

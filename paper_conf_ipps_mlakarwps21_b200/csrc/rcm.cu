@@ -9,7 +9,7 @@
 #include <new>
 
 #include "../../include/rcm.h"
-#include "rcm_workers.cuh"
+#include "rcm_lookback.cuh"
 #include "rcm_components.cuh"
 
 using namespace rcm;
@@ -135,10 +135,11 @@ __device__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemP
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) chain_init(kp, kp.chains[c]);
     grid_barrier(kp);
-    if (ld_cg_s32(&kp.ctl->status)) return;
     const uint32_t epoch = ld_acquire_u32(&kp.ctl->epoch);
     const Problem P = kp.chains[c];
     chain_worker(kp, P, sm, sh, epoch);
+    grid_barrier(kp);
+    chain_reset_signals(kp);
     grid_barrier(kp);
   }
   const int nsolo = ld_cg_s32(&kp.ctl->n_solo);
@@ -164,6 +165,8 @@ __global__ void __launch_bounds__(kThreads, 2) k_main(KParams kp, MainArgs a) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     Ctl* c = kp.ctl;
     c->ts[0] = globaltimer();
+    c->ts[5] = c->ts[6] = 0;
+    for (int i = 0; i < 8; ++i) c->dbg[i] = 0;
     c->minkey = kKeyMax; c->maxdeg = 0; c->status = 0; c->head = 0; c->done = 0; c->chain_total = 0;
     c->solo_next = 0; c->n_chain = 0; c->n_solo = 0; c->n_comp = 0; c->spill_cursor = 0; c->incomplete = 0;
     if (kp.collect_stats) *kp.stats = Stats{};
@@ -181,7 +184,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_main(KParams kp, MainArgs a) {
   if (!a.batched && a.validate == 2) validate_sym_phase(kp, a.n);
   grid_barrier(kp);
   stamp(kp, 1);
-  if (ld_cg_s32(&kp.ctl->status)) return;
+  if (ld_cg_s32(&kp.ctl->status)) return;   // read after a barrier: uniform across blocks
   if (a.gl_only) {   // rcm_find_pseudo_peripheral
     const int x = gl_phase(kp, a.w, a.n, a.gl_start, sh);
     if (gtid() == 0) *a.gl_out = x;
@@ -437,9 +440,13 @@ static int bits_for(int64_t x) {
   return b;
 }
 
+// Cooperative launch: the runtime guarantees every block of the persistent
+// grid is co-resident (grid barriers and spin-waits rely on it) or fails.
 static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& a, cudaStream_t s) {
-  k_main<<<p->nblocks, kThreads, p->smem, s>>>(kp, a);
-  CK(cudaGetLastError());
+  KParams kpc = kp;
+  MainArgs ac = a;
+  void* args[] = {&kpc, &ac};
+  CK(cudaLaunchCooperativeKernel((const void*)k_main, dim3(p->nblocks), dim3(kThreads), args, p->smem, s));
   return RCM_OK;
 }
 
@@ -537,13 +544,26 @@ extern "C" rcm_status_t rcm_get_timing(rcm_plan_t p, double* out_ms) {
   if (!p || !out_ms) return RCM_ERR_INVALID_ARGUMENT;
   unsigned long long ts[8];
   CK(cudaMemcpy(ts, p->ctl->ts, sizeof(ts), cudaMemcpyDeviceToHost));
-  // [prologue, seed + set-up, traversal, components + their traversal, total]
+  // [prologue, seed + set-up, traversal, components + their traversal, total,
+  //  component labelling, component sort + layout]
   auto d = [&](int a, int b) { return ts[b] >= ts[a] ? (double)(ts[b] - ts[a]) * 1e-6 : 0.0; };
+  const bool cc = ts[5] >= ts[3] && ts[6] >= ts[5] && ts[4] >= ts[6];
   out_ms[0] = d(0, 1);
   out_ms[1] = d(1, 2);
   out_ms[2] = d(2, 3);
   out_ms[3] = d(3, 4);
   out_ms[4] = d(0, 4);
+  out_ms[5] = cc ? d(3, 5) : 0.0;
+  out_ms[6] = cc ? d(5, 6) : 0.0;
+  return RCM_OK;
+}
+
+// Watchdog diagnostics of the last call (8 host int64): site (1 dequeue,
+// 2 look-back Discovered, 3 look-back prefix, 4 grid barrier, 5 serial chain
+// wait), slot, index, word, block.  Not part of the public header.
+extern "C" rcm_status_t rcm_debug_info(rcm_plan_t p, long long* out8) {
+  if (!p || !out8) return RCM_ERR_INVALID_ARGUMENT;
+  CK(cudaMemcpy(out8, p->ctl->dbg, 8 * sizeof(long long), cudaMemcpyDeviceToHost));
   return RCM_OK;
 }
 

@@ -31,7 +31,7 @@ struct KParams {
   int32_t nblocks;
 };
 
-enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8 };
+enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16 };
 
 // Dynamic shared memory of one worker.
 struct SmemPtrs {
@@ -76,6 +76,7 @@ struct ShState {
   int32_t t, o_begin, o_end, next;
   int32_t nP, E, steal, removed;
   int32_t s_early, s_mid, counted, aborted;
+  unsigned long long sigw;     // last signal word read from this batch's slot
   int32_t out_off, q_off, ovh_n, ovh_t;
   int32_t fwd, nb, count, chain_end;
   long long V;
@@ -90,33 +91,39 @@ __device__ __forceinline__ void latch_error(Ctl* ctl, int32_t code) {
   atomicExch(&ctl->done, 1);
 }
 
+// Watchdog expiry: record where (site) and on what, then latch RCM_ERR_HANG.
+__device__ __forceinline__ void latch_hang(Ctl* ctl, int site, long long a, long long b, long long c) {
+  if (atomicCAS(&ctl->status, 0, ST_HANG) == 0) {
+    ctl->dbg[0] = site; ctl->dbg[1] = a; ctl->dbg[2] = b; ctl->dbg[3] = c;
+    ctl->dbg[4] = blockIdx.x;
+  }
+  atomicExch(&ctl->done, 1);
+}
+
 // ---------------------------------------------------------------- signals
-__device__ __forceinline__ uint32_t load_state(const Sig* s, uint32_t epoch) {
-  unsigned long long w = ld_acquire_u64(&s->word);
-  return (uint32_t)(w >> 32) == epoch ? (uint32_t)(w & 0xffffffffu) : S_NONE;
-}
+// One acquire load returns state + payload (Sig::word).
+__device__ __forceinline__ unsigned long long load_sig(const Sig* s) { return ld_acquire_u64(&s->word); }
 
-__device__ __forceinline__ void send_state(Sig* s, uint32_t epoch, uint32_t st) {
-  __threadfence();
-  st_release_u64(&s->word, ((unsigned long long)epoch << 32) | st);
-}
+__device__ __forceinline__ void send_sig(Sig* s, unsigned long long w) { st_release_u64(&s->word, w); }
 
-// Busy wait with sleep back-off.  Returns the state, or S_NONE if
-// the chain was terminated (done) or the watchdog fired.
-__device__ uint32_t wait_state(const Sig* s, uint32_t epoch, uint32_t need, Ctl* ctl) {
-  uint32_t st = load_state(s, epoch);
-  if (st >= need) return st;
-  uint64_t t0 = globaltimer();
-  unsigned ns = 32;
-  for (;;) {
-    if (ld_relaxed_s32(&ctl->done)) return S_NONE;
-    __nanosleep(ns);
-    if (ns < 512) ns <<= 1;
-    st = load_state(s, epoch);
-    if (st >= need) return st;
-    if (globaltimer() - t0 > kWatchdogNs) {
-      latch_error(ctl, ST_HANG);
-      return S_NONE;
+// Busy wait: tight polling first, then sleep back-off.  Returns
+// the signal word, or 0 if the chain was terminated (done) or the watchdog fired.
+__device__ unsigned long long wait_sig(const Sig* s, uint32_t need, Ctl* ctl) {
+  unsigned long long w = load_sig(s);
+  if (sig_state(w) >= need) return w;
+  uint64_t t0 = 0;
+  unsigned ns = 0;
+  for (int it = 0;; ++it) {
+    if (ld_relaxed_s32(&ctl->done)) return 0;
+    if (it >= 64) {
+      __nanosleep(ns);
+      if (ns < 256) ns = ns ? ns * 2 : 32;
+    }
+    w = load_sig(s);
+    if (sig_state(w) >= need) return w;
+    if ((it & 1023) == 1023) {
+      if (t0 == 0) t0 = globaltimer();
+      else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(ctl, 5, need, (long long)w, 0); return 0; }
     }
   }
 }

@@ -8,7 +8,7 @@
 #include <cuda_runtime.h>
 
 #include "../../include/rcm.h"
-#include "rcm_workers.cuh"
+#include "rcm_lookback.cuh"
 
 namespace rcm {
 
@@ -215,6 +215,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     w.vals0[i] = v;
   }
   grid_barrier(kp);
+  stamp(kp, 5);
   int maxdeg = ld_cg_s32(&kp.ctl->maxdeg);
   int dbits = 0;
   while (dbits < 32 && (1ll << dbits) <= maxdeg) ++dbits;
@@ -273,6 +274,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     if (threadIdx.x == 0 && singles) atomicAdd(&kp.stats->components, (unsigned long long)singles);
   }
   grid_barrier(kp);
+  stamp(kp, 6);
 }
 
 // =============================================== pseudo-peripheral finder

@@ -27,16 +27,27 @@ struct __align__(16) Desc {
   uint32_t tag;
 };
 
-// Signal a batch receives from its chain predecessor:
-// word = epoch << 32 | state; payload valid once state >= S_COUNTED.
+// Signal a batch receives from its chain predecessor,
+// packed so that one acquire load returns the state AND the Counted payload:
+//   word = out_off << 33 | q_off << 3 | has_ovh << 2 | state
+//   out_off: matrix-local output position of this batch's first child (31 bit)
+//   q_off:   queue index where this batch's generated batches go (30 bit)
+//   ovh:     overhang forwarded to this batch, nodes << 32 | clamped valence
+//            sum, written before `word`, read iff has_ovh.
+// Slots are zeroed after every chain run, so 0 == S_NONE.
 struct __align__(16) Sig {
   unsigned long long word;
-  int32_t out_off;    // matrix-local output position of this batch's first child
-  int32_t q_off;      // queue index where this batch's generated batches go
-  int32_t ovh_nodes;  // overhang forwarded to this batch
-  int32_t ovh_temp;   //   ... and its (clamped) valence sum
-  int32_t pad[2];
+  unsigned long long ovh;
 };
+__host__ __device__ __forceinline__ unsigned long long sig_pack(int out_off, int q_off, int has_ovh,
+                                                                 uint32_t st) {
+  return ((unsigned long long)(uint32_t)out_off << 33) | ((unsigned long long)(uint32_t)q_off << 3) |
+         ((unsigned long long)(has_ovh & 1) << 2) | st;
+}
+__host__ __device__ __forceinline__ uint32_t sig_state(unsigned long long w) { return (uint32_t)(w & 3); }
+__host__ __device__ __forceinline__ int sig_out(unsigned long long w) { return (int)(w >> 33); }
+__host__ __device__ __forceinline__ int sig_q(unsigned long long w) { return (int)((w >> 3) & 0x3fffffffu); }
+__host__ __device__ __forceinline__ int sig_has_ovh(unsigned long long w) { return (int)((w >> 2) & 1); }
 
 // One independent unit of work: a connected component of one matrix.
 struct Problem {
@@ -71,8 +82,11 @@ struct Ctl {
   int32_t spill_cursor;        // oversize scratch allocation cursor
   int32_t chain_cur;           // chain index currently processed
   int32_t incomplete;          // 1 if the chain-first pass did not order every node
-  int32_t pad[3];
+  int32_t qtail;               // highest queue slot reserved by the current chain
+  int32_t completed;           // look-back chain: slots finished (chain-end detection)
+  int32_t pad[1];
   unsigned long long ts[8];    // phase timestamps (%globaltimer ns) of the last call
+  long long dbg[8];            // watchdog diagnostics: site, slot, index, word, ...
 };
 
 struct Stats {

@@ -1,0 +1,291 @@
+// rcm_lookback.cuh -- the default B200 chain: Alg. 5's signalling chain with
+// the two signals (Discovered, Counted) turned into per-slot status words that a
+// batch publishes about ITSELF as early as possible, and that a successor reads
+// with a decoupled look-back over a 32-slot window per round trip (one warp),
+// instead of one predecessor -> successor hand-off per batch.
+//
+//   Discovered: slot j has LOCAL once its own discovery is done and
+//     DINCL once it knows every slot <= j is discovered.  Batch t may rediscover
+//     when every slot < t is LOCAL up to the nearest DINCL slot.
+//   Counted: slot j has AGG(count_j, nb_j) once its exact
+//     output count is known (after rediscovery, before sorting -- the paper's
+//     early Counted), and INCL(out_end_j, q_end_j) once its prefix is known.
+//     Batch t's output position / queue offset = nearest INCL + sum of AGGs.
+//
+// Result-neutral: the keys, rediscovery rule and per-parent sort are those of
+// the serial chain (C-4, C-11).  Work aggregation by overhang
+// forwarding is a sequential decision and is not used here; the
+// generator batches its own outputs only.
+#pragma once
+#include "rcm_workers.cuh"
+
+namespace rcm {
+
+constexpr unsigned long long LB_LOCAL = 1, LB_DINCL = 2, LB_AGG = 4;
+
+// a-word: flags | count << 3 (31 bit) | nb << 34 (30 bit)
+__device__ __forceinline__ unsigned long long lb_a(int count, int nb, unsigned long long flags) {
+  return flags | ((unsigned long long)(uint32_t)count << 3) | ((unsigned long long)(uint32_t)nb << 34);
+}
+// b-word: INCL | out_end << 1 (31 bit) | q_end << 32
+__device__ __forceinline__ unsigned long long lb_b(int out_end, int q_end) {
+  return 1ull | ((unsigned long long)(uint32_t)out_end << 1) | ((unsigned long long)(uint32_t)q_end << 32);
+}
+
+__device__ __forceinline__ void lb_spin(unsigned& ns, int it) {
+  if (it >= 16) {
+    __nanosleep(ns);
+    if (ns < 256) ns = ns ? ns * 2 : 32;
+  }
+}
+
+// Warp 0: wait until every slot < t is discovered.  Returns false on error.
+// try_only: give up (return false, *ready = 0) instead of spinning.
+__device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int* ready) {
+  const int lane = threadIdx.x & 31;
+  int j = t - 1;
+  unsigned ns = 0;
+  uint64_t t0 = 0;
+  for (int it = 0; j >= 0; ++it) {
+    const int idx = j - lane;
+    const unsigned long long a = idx >= 0 ? ld_acquire_u64(&kp.sig[idx].word) : (LB_LOCAL | LB_DINCL);
+    const unsigned incl = __ballot_sync(0xffffffffu, (a & LB_DINCL) != 0);
+    const unsigned loc = __ballot_sync(0xffffffffu, (a & LB_LOCAL) != 0);
+    const int stop = incl ? __ffs(incl) - 1 : 32;
+    const unsigned need = stop == 32 ? 0xffffffffu : ((1u << stop) - 1);
+    if ((loc & need) == need) {
+      if (stop < 32) break;
+      j -= 32;
+      continue;
+    }
+    j -= __ffs(~loc & need) - 1;   // verified-LOCAL slots stay LOCAL (monotone)
+    if (try_only && it >= 2) { *ready = 0; return true; }
+    // A batch still waiting for Discovered has no aggregate yet, so it is a
+    // successor of the batch that completed the order (which saw every
+    // predecessor's aggregate): after early termination it has nothing to
+    // output and may be abandoned -- and must be, since a slot it waits on may
+    // have been abandoned at dequeue.
+    if (ld_relaxed_s32(&kp.ctl->status) || ld_relaxed_s32(&kp.ctl->done)) return false;
+    lb_spin(ns, it);
+    if ((it & 1023) == 1023) {
+      if (t0 == 0) t0 = globaltimer();
+      else if (globaltimer() - t0 > kWatchdogNs) { if (lane == 0) latch_hang(kp.ctl, 2, t, j, (long long)a); return false; }
+    }
+  }
+  *ready = 1;
+  return true;
+}
+
+// Warp 0: output position and queue offset of slot t (exclusive prefix).
+__device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count, int& out_off, int& q_off) {
+  const int lane = threadIdx.x & 31;
+  long long sc = 0, sn = 0;
+  int j = t - 1;
+  long long base_out = P.pos0 + 1, base_q = 1;   // the virtual predecessor of slot 0
+  unsigned ns = 0;
+  uint64_t t0 = 0;
+  for (int it = 0; j >= 0; ++it) {
+    const int idx = j - lane;
+    const bool valid = idx >= 0;
+    const unsigned long long b = valid ? ld_acquire_u64(&kp.sig[idx].ovh) : 0ull;
+    const unsigned long long a = valid ? ld_acquire_u64(&kp.sig[idx].word) : 0ull;
+    const unsigned incl = __ballot_sync(0xffffffffu, !valid || (b & 1ull));
+    const unsigned agg = __ballot_sync(0xffffffffu, valid && (a & LB_AGG));
+    const int stop = incl ? __ffs(incl) - 1 : 32;
+    const unsigned need = stop == 32 ? 0xffffffffu : ((1u << stop) - 1);
+    unsigned take = need;
+    const bool complete = (agg & need) == need;
+    if (!complete) take = (1u << (__ffs(~agg & need) - 1)) - 1;   // AGG prefix of the window
+    // accumulate the AGG lanes in `take`
+    long long c = ((take >> lane) & 1) ? (long long)((a >> 3) & 0x7fffffffull) : 0;
+    long long q = ((take >> lane) & 1) ? (long long)(a >> 34) : 0;
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+      c += __shfl_xor_sync(0xffffffffu, c, d);
+      q += __shfl_xor_sync(0xffffffffu, q, d);
+    }
+    sc += c;
+    sn += q;
+    if (complete) {
+      if (stop < 32) {
+        const unsigned long long bs = __shfl_sync(0xffffffffu, b, stop);
+        const int vs = __shfl_sync(0xffffffffu, (int)valid, stop);
+        if (vs) { base_out = (long long)((bs >> 1) & 0x7fffffffull); base_q = (long long)(bs >> 32); }
+        j = -1;
+        break;
+      }
+      j -= 32;
+      continue;
+    }
+    j -= __popc(take);
+    // after early termination only batches without output may give up (a batch
+    // with output precedes the terminating batch, whose look-back saw all of
+    // its predecessors' aggregates, so this loop finishes)
+    if (ld_relaxed_s32(&kp.ctl->status) || (count == 0 && ld_relaxed_s32(&kp.ctl->done))) return false;
+    lb_spin(ns, it);
+    if ((it & 1023) == 1023) {
+      if (t0 == 0) t0 = globaltimer();
+      else if (globaltimer() - t0 > kWatchdogNs) { if (lane == 0) latch_hang(kp.ctl, 3, t, j, (long long)a); return false; }
+    }
+  }
+  out_off = (int)(base_out + sc);
+  q_off = (int)(base_q + sn);
+  return true;
+}
+
+__device__ __forceinline__ int lb_nb(const KParams& kp, int N, long long V) {
+  if (N <= 0) return 0;
+  // safe over-estimate of the greedy batch count
+  const long long v2 = (2 * V + kp.T - 1) / kp.T;
+  return N / kp.BS + (int)(v2 > 1 ? v2 : 1);
+}
+
+// Process one dequeued batch with the look-back chain.
+__device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                         uint32_t epoch) {
+  const int t = sh.t, o_begin = sh.o_begin;
+  Sig* mine = kp.sig + t;
+  const int nP = load_parents(kp, P, sm, sh, o_begin, sh.o_end - o_begin, false);
+  const int E = sh.E;
+  const bool oversize = E > kp.T;
+  const uint32_t key0 = (uint32_t)o_begin + 1;
+  if (threadIdx.x == 0) { sh.steal = 0; sh.aborted = 0; sh.s_early = 0; }
+  __syncthreads();
+  if (oversize) {
+    if (!oversize_discover(kp, P, sm, sh, key0, sm.p_rs[0], E)) return;
+  } else {
+    discover(kp, P, sm, sh, o_begin, nP, E);
+  }
+  if (threadIdx.x == 0) {                       // own discovery done: LOCAL
+    __threadfence();                            // the block's atomicMin marks first
+    st_release_u64(&mine->word, LB_LOCAL);
+  }
+  // early Discovered: all predecessors already discovered?
+  if (threadIdx.x < 32 && !oversize && !(kp.flags & F_NO_EARLY)) {
+    int ready = 0;
+    if (!lb_wait_discovered(kp, t, true, &ready)) ready = -1;
+    if (threadIdx.x == 0) { sh.s_early = ready; if (ready < 0) sh.aborted = 1; }
+  }
+  __syncthreads();
+  if (sh.aborted) return;
+  const bool early = sh.s_early == 1;
+  if (early) {
+    if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
+    rediscover(kp, P, sm, sh, o_begin, E);      // dense array after sorting
+    count_outputs(kp, sm, sh, nP, E);
+    if (threadIdx.x == 0) {
+      sh.nb = lb_nb(kp, sh.count, sh.V);
+      st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));   // early Counted
+      stat_add(kp, &kp.stats->redisc_early, 1);
+    }
+    if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
+  } else {
+    if (!oversize && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // speculative sort
+    if (threadIdx.x < 32) {
+      int ready = 0;
+      if (!lb_wait_discovered(kp, t, false, &ready) && threadIdx.x == 0) sh.aborted = 1;
+    }
+    __syncthreads();
+    if (sh.aborted) return;
+    if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
+    if (oversize) {
+      oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
+    } else {
+      const int removed = rediscover(kp, P, sm, sh, o_begin, E);
+      if (removed && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
+      count_outputs(kp, sm, sh, nP, E);
+    }
+    if (threadIdx.x == 0) {
+      sh.nb = lb_nb(kp, sh.count, sh.V);
+      st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));
+      stat_add(kp, &kp.stats->redisc_late, 1);
+    }
+  }
+  // Counted: prefix over the predecessors' aggregates
+  if (threadIdx.x < 32) {
+    int out_off = 0, q_off = 0;
+    const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off);
+    if (threadIdx.x == 0) {
+      if (!ok) {
+        sh.aborted = 1;
+      } else {
+        sh.out_off = out_off;
+        sh.q_off = q_off;
+        if ((long long)q_off + sh.nb > kp.qcap) { latch_error(kp.ctl, ST_CAPACITY); sh.nb = 0; sh.aborted = 1; }
+        st_release_u64(&mine->ovh, lb_b(out_off + sh.count, q_off + sh.nb));
+        atomicMax(&kp.ctl->qtail, q_off + sh.nb);
+        atomicMax(&kp.ctl->chain_total, out_off + sh.count);
+        stat_add(kp, &kp.stats->generated, sh.nb);
+      }
+    }
+  }
+  __syncthreads();
+  if (sh.aborted) return;
+  const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
+  GenState g;
+  if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; }
+  if (oversize) {
+    if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) return;
+    oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
+    if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
+  } else {
+    if (kp.flags & F_NO_SORT) compact_segments(sm, sh, nP);
+    write_output(kp, P, sm, sh, nP, E, out_off);
+    __threadfence();
+    __syncthreads();
+    if (nb > 0) {
+      build_prefix(kp, sm, sh, E);
+      if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
+    }
+  }
+  if (threadIdx.x == 0) {
+    if (nb > 0) {
+      gen_finish(kp, g, out_off + sh.count, q_off, nb, epoch);
+      if (g.emitted > nb) latch_error(kp.ctl, ST_CAPACITY);
+    }
+    sh.k = nb > 0 ? g.emitted : 0;
+    stat_add(kp, &kp.stats->executed, 1);
+  }
+  __syncthreads();
+  // empty slots: published as discovered with a zero aggregate
+  const int emitted = sh.k;
+  if (nb > emitted && threadIdx.x < 32) {
+    for (int i = emitted + threadIdx.x; i < nb; i += 32) {
+      st_release_u64(&kp.sig[q_off + i].word, LB_LOCAL | LB_AGG);
+      publish_desc(kp.desc + q_off + i, 0, 0, q_off + i + 1, epoch);
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const int total = out_off + sh.count;
+    if (total == P.pos0 + P.size) {             // early termination
+      __threadfence();
+      atomicExch(&kp.ctl->done, 1);
+    } else {
+      // chain end: every reserved slot finished (each slot reserves before it
+      // counts itself; empties are counted by their generator)
+      __threadfence();
+      const int c = atomicAdd(&kp.ctl->completed, 1 + (nb - emitted)) + 1 + (nb - emitted);
+      if (c == ld_acquire_s32(&kp.ctl->qtail)) {
+        kp.ctl->incomplete = 1;
+        __threadfence();
+        atomicExch(&kp.ctl->done, 1);
+      }
+    }
+  }
+  __syncthreads();
+}
+
+__device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                             uint32_t epoch) {
+  for (;;) {
+    if (threadIdx.x == 0) sh.aborted = dequeue(kp, sh, epoch) ? 0 : 1;
+    __syncthreads();
+    if (sh.aborted) break;
+    if (kp.flags & F_SERIAL_CHAIN) chain_batch(kp, P, sm, sh, epoch);   // Alg. 5 hand-off chain
+    else lb_batch(kp, P, sm, sh, epoch);                                 // look-back chain
+  }
+  __syncthreads();
+}
+
+}  // namespace rcm

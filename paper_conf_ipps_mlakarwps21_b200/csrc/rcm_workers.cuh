@@ -35,8 +35,8 @@ __device__ void grid_barrier(const KParams& kp) {
     } else {
       uint64_t t0 = globaltimer();
       while (ld_acquire_s32(&kp.ctl->gbar_gen) == gen) {
-        __nanosleep(128);
-        if (globaltimer() - t0 > kWatchdogNs) { latch_error(kp.ctl, ST_HANG); break; }
+        __nanosleep(64);
+        if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 4, gen, 0, 0); break; }
       }
     }
   }
@@ -299,14 +299,19 @@ __device__ void oversize_output(const KParams& kp, const Problem& P, const SmemP
 
 // ------------------------------------------------------------ chain worker
 // signalCount (Alg. 5 ln 31-40): with the exact output count known
-// and the predecessor's output position received, forward the position, the
-// queue offset and possibly an overhang to the successor.  Thread 0 only.
-__device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, Sig* succ_sig,
-                             int succ, uint32_t epoch) {
-  const int out_off = ld_relaxed_s32(&mine->out_off);
-  const int q_off = ld_relaxed_s32(&mine->q_off);
-  const int ovh_n = ld_relaxed_s32(&mine->ovh_nodes);
-  const int ovh_t = ld_relaxed_s32(&mine->ovh_temp);
+// and the predecessor's output position received (signal word `w`), forward the
+// position, the queue offset and possibly an overhang to the successor.
+// Thread 0 only.
+__device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, unsigned long long w,
+                             Sig* succ_sig, int succ) {
+  const int out_off = sig_out(w);
+  const int q_off = sig_q(w);
+  int ovh_n = 0, ovh_t = 0;
+  if (sig_has_ovh(w)) {
+    const unsigned long long ov = ld_relaxed_u64(&mine->ovh);   // ordered after the acquire of w
+    ovh_n = (int)(ov >> 32);
+    ovh_t = (int)(uint32_t)ov;
+  }
   const int Np = ovh_n + sh.count;
   const long long Vp = (long long)ovh_t + sh.V;
   // combine with next: below half a batch in nodes and temp
@@ -315,30 +320,26 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, Si
                    2 * Vp < (long long)kp.T && succ < q_off;
   int nb = 0;
   if (fwd) {
-    st_relaxed_s32(&succ_sig->out_off, out_off + sh.count);
-    st_relaxed_s32(&succ_sig->q_off, q_off);
-    st_relaxed_s32(&succ_sig->ovh_nodes, Np);
-    st_relaxed_s32(&succ_sig->ovh_temp, (int)Vp);
-    send_state(succ_sig, epoch, S_COUNTED);
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(&succ_sig->ovh),
+                 "l"(((unsigned long long)(uint32_t)Np << 32) | (uint32_t)Vp) : "memory");
+    send_sig(succ_sig, sig_pack(out_off + sh.count, q_off, 1, S_COUNTED));
     stat_add(kp, &kp.stats->ovh_forwards, 1);
   } else {
     if (Np > 0) {
       // safe over-estimate of the greedy batch count:
       // floor(N/B_s) + max(1, ceil(2V/T))  (P:L800-809 uses 2x the ideal count)
-      long long v2 = (2 * Vp + kp.T - 1) / kp.T;
+      const long long v2 = (2 * Vp + kp.T - 1) / kp.T;
       nb = Np / kp.BS + (int)(v2 > 1 ? v2 : 1);
     }
     if ((long long)q_off + nb > kp.qcap) {
       latch_error(kp.ctl, ST_CAPACITY);
       nb = 0;
     }
-    st_relaxed_s32(&succ_sig->out_off, out_off + sh.count);
-    st_relaxed_s32(&succ_sig->q_off, q_off + nb);
-    st_relaxed_s32(&succ_sig->ovh_nodes, 0);
-    st_relaxed_s32(&succ_sig->ovh_temp, 0);
-    send_state(succ_sig, epoch, S_COMPLETED);   // nothing to wait for (Alg. 5 ln 39)
+    send_sig(succ_sig, sig_pack(out_off + sh.count, q_off + nb, 0, S_COMPLETED));  // Alg. 5 ln 39
+    if (nb) atomicMax(&kp.ctl->qtail, q_off + nb);
     stat_add(kp, &kp.stats->generated, nb);
   }
+  sh.sigw = w;
   sh.out_off = out_off;
   sh.q_off = q_off;
   sh.ovh_n = ovh_n;
@@ -354,22 +355,26 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, Si
 __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
   for (;;) {
     if (ld_relaxed_s32(&kp.ctl->done)) return false;
-    int t = atomicAdd(&kp.ctl->head, 1);
+    const int t = atomicAdd(&kp.ctl->head, 1);
     if (t >= kp.qcap) {   // only possible after a capacity error; wait for done
       while (!ld_relaxed_s32(&kp.ctl->done)) __nanosleep(1000);
       return false;
     }
     const Desc* d = kp.desc + t;
     uint64_t t0 = 0;
-    unsigned ns = 32;
-    while (ld_acquire_u32(&d->tag) != epoch) {
+    unsigned ns = 0;
+    for (int it = 0; ld_acquire_u32(&d->tag) != epoch; ++it) {
       if (ld_relaxed_s32(&kp.ctl->done)) return false;
-      if (t0 == 0) t0 = globaltimer();
-      __nanosleep(ns);
-      if (ns < 256) ns <<= 1;
-      if (globaltimer() - t0 > kWatchdogNs) { latch_error(kp.ctl, ST_HANG); return false; }
+      if (it >= 32) {
+        __nanosleep(ns);
+        if (ns < 512) ns = ns ? ns * 2 : 32;
+      }
+      if ((it & 255) == 255) {
+        if (t0 == 0) t0 = globaltimer();
+        else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 1, t, ld_relaxed_s32(&kp.ctl->head), 0); return false; }
+      }
     }
-    int b = ld_relaxed_s32(&d->o_begin), e = ld_relaxed_s32(&d->o_end), nx = ld_relaxed_s32(&d->next);
+    const int b = ld_relaxed_s32(&d->o_begin), e = ld_relaxed_s32(&d->o_end), nx = ld_relaxed_s32(&d->next);
     stat_add(kp, &kp.stats->dequeued, 1);
     if (b == e) { stat_add(kp, &kp.stats->empty, 1); continue; }
     sh.t = t;
@@ -392,7 +397,7 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
     sh.steal = 0;
     sh.counted = 0;
     sh.aborted = 0;
-    sh.s_early = (kp.flags & F_NO_EARLY) ? S_NONE : load_state(mine, epoch);   // ln 2
+    sh.s_early = (kp.flags & F_NO_EARLY) ? S_NONE : sig_state(load_sig(mine));   // ln 2
   }
   __syncthreads();
   const bool oversize = E > kp.T;   // only single-node batches (batch generation)
@@ -400,53 +405,61 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
   if (oversize) {
     if (!oversize_discover(kp, P, sm, sh, key0, sm.p_rs[0], E)) return;
   } else {
-    discover(kp, P, sm, sh, o_begin, nP, E);                                   // ln 3
+    discover(kp, P, sm, sh, o_begin, nP, E);                                    // ln 3
   }
-  if (threadIdx.x == 0) sh.s_mid = load_state(mine, epoch);                    // ln 4
+  if (threadIdx.x == 0) { sh.sigw = load_sig(mine); sh.s_mid = sig_state(sh.sigw); }  // ln 4
   __syncthreads();
   const int s_early = sh.s_early, s_mid = sh.s_mid;
   bool rediscovered = false;
   if (!oversize && (s_early >= S_DISCOVERED || s_mid >= S_DISCOVERED)) {
     // ln 5-12: every predecessor has discovered; forward Discovered right after
     // our own discovery, rediscover before sorting (dense array after sorting).
-    if (threadIdx.x == 0) send_state(succ_sig, epoch, S_DISCOVERED);
+    if (threadIdx.x == 0) {
+      __threadfence();   // the block's atomicMin marks before the signal
+      send_sig(succ_sig, S_DISCOVERED);
+    }
     if (s_early < S_DISCOVERED || sh.steal) {
       rediscover(kp, P, sm, sh, o_begin, E);
       if (threadIdx.x == 0 && s_early < S_DISCOVERED) stat_add(kp, &kp.stats->redisc_early, 1);
     }
     rediscovered = true;
     count_outputs(kp, sm, sh, nP, E);
-    if (threadIdx.x == 0 && s_mid >= S_COUNTED) signal_count(kp, sh, mine, succ_sig, succ, epoch);
+    if (threadIdx.x == 0) {
+      const unsigned long long w = load_sig(mine);
+      if (sig_state(w) >= S_COUNTED) signal_count(kp, sh, mine, w, succ_sig, succ);
+    }
     __syncthreads();
   }
   if (!oversize) {
-    if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);               // ln 13
+    if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);                // ln 13
   }
   if (!rediscovered) {
     // ln 14-19: late discovery -- wait for Discovered, forward it, rediscover
     if (threadIdx.x == 0) {
-      if (wait_state(mine, epoch, S_DISCOVERED, kp.ctl) < S_DISCOVERED) sh.aborted = 1;
-      else send_state(succ_sig, epoch, S_DISCOVERED);
+      if (sig_state(wait_sig(mine, S_DISCOVERED, kp.ctl)) < S_DISCOVERED) sh.aborted = 1;
+      else { __threadfence(); send_sig(succ_sig, S_DISCOVERED); }
     }
     __syncthreads();
     if (sh.aborted) return;
     if (oversize) {
       oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
     } else {
-      int removed = rediscover(kp, P, sm, sh, o_begin, E);
+      const int removed = rediscover(kp, P, sm, sh, o_begin, E);
       if (removed && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // move removed to the end
       count_outputs(kp, sm, sh, nP, E);
     }
     if (threadIdx.x == 0) {
       stat_add(kp, &kp.stats->redisc_late, 1);
-      if (load_state(mine, epoch) >= S_COUNTED) signal_count(kp, sh, mine, succ_sig, succ, epoch);
+      const unsigned long long w = load_sig(mine);
+      if (sig_state(w) >= S_COUNTED) signal_count(kp, sh, mine, w, succ_sig, succ);
     }
     __syncthreads();
   }
-  if (!sh.counted) {                                                           // ln 20-22
+  if (!sh.counted) {                                                            // ln 20-22
     if (threadIdx.x == 0) {
-      if (wait_state(mine, epoch, S_COUNTED, kp.ctl) < S_COUNTED) sh.aborted = 1;
-      else signal_count(kp, sh, mine, succ_sig, succ, epoch);
+      const unsigned long long w = wait_sig(mine, S_COUNTED, kp.ctl);
+      if (sig_state(w) < S_COUNTED) sh.aborted = 1;
+      else signal_count(kp, sh, mine, w, succ_sig, succ);
     }
     __syncthreads();
     if (sh.aborted) return;
@@ -462,12 +475,13 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
     g.has_pend = 0;
   }
   const bool gen = !sh.fwd && sh.nb > 0;
+  // wait(Completed) before publishing batches that reference an overhang, or
+  // before forwarding Completed for an overhang we passed on (ln 27-29)
+  const bool need_completed = sh.fwd || sh.ovh_n > 0;
   if (oversize) {
-    if (kp.flags & F_NO_SORT) { /* sorting disabled has no effect on the single-parent path */ }
     if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) return;
-    // wait(Completed) before publishing batches that reference an overhang
-    if (threadIdx.x == 0 && (sh.fwd || sh.ovh_n > 0)) {
-      if (wait_state(mine, epoch, S_COMPLETED, kp.ctl) < S_COMPLETED) sh.aborted = 1;
+    if (threadIdx.x == 0 && need_completed && sig_state(sh.sigw) < S_COMPLETED) {
+      if (sig_state(wait_sig(mine, S_COMPLETED, kp.ctl)) < S_COMPLETED) sh.aborted = 1;
     }
     __syncthreads();
     if (sh.aborted) return;
@@ -478,9 +492,8 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
     write_output(kp, P, sm, sh, nP, E, out_off);
     __threadfence();
     __syncthreads();
-    // ln 27-29: wait(Completed); if we forwarded an overhang, signal Completed
-    if (threadIdx.x == 0 && (sh.fwd || sh.ovh_n > 0)) {
-      if (wait_state(mine, epoch, S_COMPLETED, kp.ctl) < S_COMPLETED) sh.aborted = 1;
+    if (threadIdx.x == 0 && need_completed && sig_state(sh.sigw) < S_COMPLETED) {
+      if (sig_state(wait_sig(mine, S_COMPLETED, kp.ctl)) < S_COMPLETED) sh.aborted = 1;
     }
     __syncthreads();
     if (sh.aborted) return;
@@ -490,9 +503,9 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
     }
   }
   if (threadIdx.x == 0) {
-    if (sh.fwd) send_state(succ_sig, epoch, S_COMPLETED);
+    if (sh.fwd) send_sig(succ_sig, sig_pack(out_off + sh.count, sh.q_off, 1, S_COMPLETED));
     if (gen) {
-      gen_finish(kp, g, out_off + sh.count, sh.q_off, sh.nb, epoch);          // ln 30
+      gen_finish(kp, g, out_off + sh.count, sh.q_off, sh.nb, epoch);           // ln 30
       if (g.emitted > sh.nb) latch_error(kp.ctl, ST_CAPACITY);
     }
     sh.k = gen ? g.emitted : 0;
@@ -520,16 +533,16 @@ __device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs&
 // predecessor is Completed with out_off = pos0+1 and queue tail 1.  Thread 0 of
 // block 0, before a grid barrier.
 __device__ void chain_init(const KParams& kp, const Problem& P) {
-  uint32_t ep = atomicAdd(&kp.ctl->epoch, 1u) + 1u;
+  const uint32_t ep = atomicAdd(&kp.ctl->epoch, 1u) + 1u;
   kp.ctl->head = 0;
   kp.ctl->done = 0;
+  kp.ctl->qtail = 1;
+  kp.ctl->completed = 0;
   place_root(kp, P, P.seed, P.pos0);
-  Sig* s0 = kp.sig;
-  s0->out_off = P.pos0 + 1;
-  s0->q_off = 1;
-  s0->ovh_nodes = 0;
-  s0->ovh_temp = 0;
-  s0->word = ((unsigned long long)ep << 32) | S_COMPLETED;
+  kp.sig[0].ovh = 0;
+  // serial chain: the virtual predecessor of slot 0 has Completed with
+  // out_off = pos0+1 and queue tail 1; look-back chain: slot 0 starts empty
+  kp.sig[0].word = (kp.flags & F_SERIAL_CHAIN) ? sig_pack(P.pos0 + 1, 1, 0, S_COMPLETED) : 0ull;
   Desc* d0 = kp.desc;
   d0->o_begin = P.pos0;
   d0->o_end = P.pos0 + 1;
@@ -539,15 +552,14 @@ __device__ void chain_init(const KParams& kp, const Problem& P) {
   __threadfence();
 }
 
-__device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
-                             uint32_t epoch) {
-  for (;;) {
-    if (threadIdx.x == 0) sh.aborted = dequeue(kp, sh, epoch) ? 0 : 1;
-    __syncthreads();
-    if (sh.aborted) break;
-    chain_batch(kp, P, sm, sh, epoch);
+// After a chain run (all blocks, between grid barriers): zero the signal slots
+// it used so the next run starts from S_NONE without an epoch in the word.
+__device__ void chain_reset_signals(const KParams& kp) {
+  const int qt = min(ld_cg_s32(&kp.ctl->qtail) + 2, kp.qcap + 1);
+  for (int i = blockIdx.x * kThreads + threadIdx.x; i < qt; i += kp.nblocks * kThreads) {
+    kp.sig[i].word = 0;
+    kp.sig[i].ovh = 0;
   }
-  __syncthreads();
 }
 
 // ------------------------------------------------------------- solo worker

@@ -56,10 +56,12 @@ def _tiny_graphs():
 MODES = [(oracle.FIXED, "mid"), (oracle.MIN_DEGREE, None)]
 PATHS = {
     "solo": dict(),
-    "chain": dict(flags=8, solo_threshold=-1),
+    "chain": dict(flags=8, solo_threshold=-1),                       # look-back chain (default)
     "chain_bs1": dict(flags=8, solo_threshold=-1, batch_nodes=1),
-    "chain_bs3_noovh": dict(flags=8 | 1, solo_threshold=-1, batch_nodes=3),
     "chain_noearly": dict(flags=8 | 2, solo_threshold=-1, batch_nodes=7, temp_elems=2304),
+    "serial": dict(flags=8 | 16, solo_threshold=-1),                 # Alg. 5 hand-off chain
+    "serial_bs3_noovh": dict(flags=8 | 16 | 1, solo_threshold=-1, batch_nodes=3),
+    "serial_noearly": dict(flags=8 | 16 | 2, solo_threshold=-1, batch_nodes=7, temp_elems=2304),
 }
 
 
@@ -74,7 +76,7 @@ def test_tiny_families(rcm, path):
 
 
 @pytest.mark.parametrize("cfg", [1, 2, 3, 4])
-@pytest.mark.parametrize("path", ["solo", "chain", "chain_bs3_noovh"])
+@pytest.mark.parametrize("path", ["solo", "chain", "serial", "serial_bs3_noovh"])
 def test_config_small_twins(rcm, cfg, path):
     g, mode, start = synth.config_graph(cfg, "small")
     ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
@@ -88,7 +90,8 @@ def test_config_small_twins(rcm, cfg, path):
 @pytest.mark.parametrize("opts", [
     dict(batch_nodes=1), dict(batch_nodes=2), dict(batch_nodes=3), dict(batch_nodes=64),
     dict(batch_nodes=1024), dict(temp_elems=2304), dict(blocks_per_sm=1), dict(flags=1), dict(flags=2),
-    dict(flags=3, batch_nodes=16, temp_elems=2304),
+    dict(flags=3, batch_nodes=16, temp_elems=2304), dict(flags=16), dict(flags=16, batch_nodes=1),
+    dict(flags=16 | 1), dict(flags=16 | 2), dict(flags=16, blocks_per_sm=1, batch_nodes=1024),
 ])
 def test_sweep_invariance(rcm, opts):
     g, mode, start = synth.config_graph(2, "small")
@@ -103,8 +106,10 @@ def test_repeat_determinism_and_stats(rcm):
     g, mode, start = synth.config_graph(2, "small")
     ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
     plan = rcm.Plan(g.n, g.nnz, solo_threshold=-1, collect_stats=1, batch_nodes=64)
+    plan2 = rcm.Plan(g.n, g.nnz, solo_threshold=-1, collect_stats=1, batch_nodes=64, flags=16)
     rp, ci = _dev(g)
-    for _ in range(30):
+    for it in range(40):
+        plan, plan2 = plan2, plan
         perm = plan.reorder(rp, ci, mode, start).cpu().numpy()
         assert np.array_equal(perm, ref)
         st = plan.stats()
@@ -113,6 +118,7 @@ def test_repeat_determinism_and_stats(rcm):
         assert st["batches_executed"] + st["batches_empty"] <= st["batches_dequeued"]
         assert st["components"] == 1
     plan.close()
+    plan2.close()
 
 
 @pytest.mark.parametrize("cfg", [1, 2])

@@ -7,13 +7,19 @@ import torch
 import oracle, synth
 import paper_conf_ipps_mlakarwps21_b200 as rcm
 
+import ctypes
+_lib = rcm._load()
+_lib.rcm_debug_info.argtypes = [ctypes.c_void_p, ctypes.POINTER(ctypes.c_longlong)]
+
 def run(g, mode, start, **opts):
     plan = rcm.Plan(max(g.n, 1), max(g.nnz, 1), collect_stats=1, **opts)
     rp = torch.from_numpy(g.row_ptr).cuda(); ci = torch.from_numpy(g.col_idx).cuda()
     try:
         perm = plan.reorder(rp, ci, mode, start).cpu().numpy()
     except Exception as e:
-        return None, str(e)
+        a = (ctypes.c_longlong * 8)()
+        _lib.rcm_debug_info(plan.handle, a)
+        return None, str(e) + " dbg=" + str(list(a)) + " stats=" + str(plan.stats())
     st = plan.stats(); plan.close()
     return perm, st
 
