@@ -202,7 +202,7 @@ __global__ void __launch_bounds__(kThreads, 2) k_main(KParams kp, MainArgs a) {
     }
     if (gtid() == 0) { a.w.sctl[0] = a.num_mats; a.w.sctl[1] = 0; }
     grid_barrier(kp);
-    radix_sort_phase(kp, a.w, 64, reinterpret_cast<int32_t*>(sm.cand), sh);
+    radix_sort_phase(kp, a.w, 0, 64, reinterpret_cast<int32_t*>(sm.cand), sh);
     const int32_t* order = ld_cg_s32(a.w.sctl + 1) ? a.w.vals1 : a.w.vals0;
     Problem* solos = const_cast<Problem*>(kp.solos);
     for (int i = gtid(); i < a.num_mats; i += G) {
@@ -353,6 +353,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_main, kThreads, p->smem);
   if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
   p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
+  if (p->nblocks > kThreads) p->nblocks = kThreads / p->num_sms * p->num_sms;   // block-0 scans assume <= kThreads
   // queue bound: sum over generating batches of floor(N/B) + max(1, ceil(2V/T))
   const int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
   p->qcap = o.queue_capacity ? o.queue_capacity : std::min<int64_t>(qb, (1ll << 31) - 2);
@@ -378,7 +379,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   AL(p->spill, 8 * 2 * p->spill_cap);
   AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
   AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
-  AL(p->w.offs, 8 * (n + 1)); AL(p->w.hist, 4 * 256 * tiles); AL(p->w.sctl, 4 * 64);
+  AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kThreads)); AL(p->w.sctl, 4 * 64);
   AL(p->w.order, 4 * n); AL(p->w.lev, 4 * n); AL(p->w.front0, 4 * n); AL(p->w.front1, 4 * n);
   AL(p->w.gctl, 4 * 64); AL(p->w.gkey, 8 * 64);
 #undef AL

@@ -67,10 +67,11 @@ __device__ __forceinline__ void stamp(const KParams& kp, int i) {
 }
 
 // ============================================================ radix sort
-// Grid-wide stable LSD radix sort of (key, val) pairs by the low `nbits` bits
-// (8-bit digits).  Count in w.sctl[0]; w.sctl[1] = buffer holding the data.
+// Grid-wide stable LSD radix sort of (key, val) pairs by bits [lo_bit, hi_bit)
+// (8-bit digits; the order of equal keys -- and thus of bits below lo_bit when
+// the input is already ordered by them -- is preserved).  Count in w.sctl[0]; w.sctl[1] = buffer holding the data.
 // A digit that is equal in all keys is skipped.  `scratch`: >= 17 KB smem.
-__device__ void radix_sort_phase(const KParams& kp, const CompWS& w, int nbits, int32_t* scratch,
+__device__ void radix_sort_phase(const KParams& kp, const CompWS& w, int lo_bit, int hi_bit, int32_t* scratch,
                                  ShState& sh) {
   const int count = ld_cg_s32(w.sctl);
   if (count <= 1) return;
@@ -79,7 +80,7 @@ __device__ void radix_sort_phase(const KParams& kp, const CompWS& w, int nbits, 
   const unsigned lt = (1u << lane) - 1;
   int32_t* off = scratch;           // 256
   int32_t* wcnt = scratch + 256;    // kWarps x 256
-  for (int shift = 0; shift < nbits; shift += 8) {
+  for (int shift = lo_bit; shift < hi_bit; shift += 8) {
     const int cur = ld_cg_s32(w.sctl + 1);
     const unsigned long long* sk = cur ? w.keys1 : w.keys0;
     const int32_t* sv = cur ? w.vals1 : w.vals0;
@@ -169,10 +170,29 @@ __device__ __forceinline__ int uf_find(int32_t* label, int x) {
   return x;
 }
 
+// Union two nodes: hook the larger root under the smaller (ECL-CC style).
+__device__ __forceinline__ void uf_unite(int32_t* label, int u, int c) {
+  for (;;) {
+    int x = uf_find(label, u), y = uf_find(label, c);
+    if (x == y) return;
+    if (x > y) { int t = x; x = y; y = t; }
+    if (atomicCAS(label + y, y, x) == y) return;
+  }
+}
+
+// Grid-wide ordered scan helper: block b owns [b*C, min(n,(b+1)*C)).
+__device__ __forceinline__ void chunk_of(const KParams& kp, long long n, long long& b, long long& e) {
+  const long long C = (n + kp.nblocks - 1) / kp.nblocks;
+  b = min(n, (long long)blockIdx.x * C);
+  e = min(n, b + C);
+}
+
 __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
   const CompWS& w = a.w;
   const int n = a.n;
   const int G = gthreads(kp);
+  const int lane = threadIdx.x & 31;
+  const int gwarp = gtid() >> 5, nwarps = G >> 5;
   // init
   for (int v = gtid(); v < n; v += G) {
     const bool unv = (uint32_t)(ld_relaxed_u64(kp.word + v) >> 32) == kInf;
@@ -180,59 +200,141 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     w.ckey[v] = kKeyMax;
     w.csize[v] = 0;
   }
-  if (gtid() == 0) { w.sctl[0] = 0; w.sctl[1] = 0; }
+  if (gtid() == 0) { w.gctl[1] = 0; w.gctl[2] = 0; }
   grid_barrier(kp);
-  // hook
+  // hook every edge (c < u: the pattern is symmetric) -- thread / warp / block
+  // per row by degree so that hub rows are split across many threads; rows
+  // above 32 entries are listed during the thread pass (front0 / front1)
   for (int u = gtid(); u < n; u += G) {
+    const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
     if (ld_cg_s32(w.label + u) < 0) continue;
-    for (int e = __ldg(kp.row_ptr + u); e < __ldg(kp.row_ptr + u + 1); ++e) {
+    if (re - rs > 32) {
+      if (re - rs > 4096) w.front1[atomicAdd(w.gctl + 2, 1)] = u;
+      else w.front0[atomicAdd(w.gctl + 1, 1)] = u;
+      continue;
+    }
+    for (int e = rs; e < re; ++e) {
       const int c = __ldg(kp.col_idx + e);
-      if (c == u || ld_cg_s32(w.label + c) < 0) continue;
-      for (;;) {
-        int x = uf_find(w.label, u), y = uf_find(w.label, c);
-        if (x == y) break;
-        if (x > y) { int t = x; x = y; y = t; }
-        if (atomicCAS(w.label + y, y, x) == y) break;
-      }
+      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
     }
   }
   grid_barrier(kp);
-  // compress + per-root key and size
-  for (int v = gtid(); v < n; v += G) {
-    if (ld_cg_s32(w.label + v) < 0) continue;
-    const int r = uf_find(w.label, v);
-    const unsigned long long k = ((ld_relaxed_u64(kp.word + v) & 0xffffffffull) << 32) | (uint32_t)v;
-    atomicMin(w.ckey + r, k);
-    atomicAdd(w.csize + r, 1);
+  const int nmed = ld_cg_s32(w.gctl + 1), nbig = ld_cg_s32(w.gctl + 2);
+  for (int i = gwarp; i < nmed; i += nwarps) {
+    const int u = __ldcg(w.front0 + i);
+    const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
+    for (int e = rs + lane; e < re; e += 32) {
+      const int c = __ldg(kp.col_idx + e);
+      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
+    }
+  }
+  for (int i = blockIdx.x; i < nbig; i += kp.nblocks) {
+    const int u = __ldcg(w.front1 + i);
+    const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
+    for (int e = rs + threadIdx.x; e < re; e += kThreads) {
+      const int c = __ldg(kp.col_idx + e);
+      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
+    }
   }
   grid_barrier(kp);
-  // collect roots as (compact key, root); the list order is fixed by the sort
-  for (int v = gtid(); v < n; v += G) {
-    if (ld_cg_s32(w.label + v) != v) continue;
-    const int i = atomicAdd(w.sctl, 1);
-    const unsigned long long k = __ldcg(w.ckey + v);
-    w.keys0[i] = ((k >> 32) << a.idbits) | (k & 0xffffffffull);
-    w.vals0[i] = v;
+  // compress; per root: minimum (valence, id) member and size
+  // warp-aggregated per root: the giant component's nodes would otherwise all
+  // hit one address with atomics
+  for (int base = blockIdx.x * kThreads; base < n; base += G) {
+    const int v = base + threadIdx.x;
+    int r = -1;
+    unsigned long long k = kKeyMax;
+    if (v < n && ld_cg_s32(w.label + v) >= 0) {
+      r = uf_find(w.label, v);
+      w.label[v] = r;
+      k = ((ld_relaxed_u64(kp.word + v) & 0xffffffffull) << 32) | (uint32_t)v;
+    }
+    const unsigned peers = __match_any_sync(0xffffffffu, r);
+    unsigned long long m;
+    int cnt;
+    {   // reduce over the peer group (lanes with the same root)
+      unsigned rest = peers;
+      unsigned long long mm = kKeyMax;
+      while (rest) {
+        const int l = __ffs(rest) - 1;
+        rest &= rest - 1;
+        const unsigned long long x = __shfl_sync(peers, k, l);
+        mm = x < mm ? x : mm;
+      }
+      m = mm;
+      cnt = __popc(peers);
+    }
+    if (r >= 0 && lane == __ffs(peers) - 1) {
+      atomicMin(w.ckey + r, m);
+      atomicAdd(w.csize + r, cnt);
+    }
+  }
+  grid_barrier(kp);
+  // ordered compaction of component representatives (the min (valence, id)
+  // member): the list comes out in id order, so a stable sort on the valence
+  // bits alone yields (valence, id) order (C-6)
+  long long cb, ce;
+  chunk_of(kp, n, cb, ce);
+  {
+    int cnt = 0;
+    for (long long v = cb + threadIdx.x; v < ce; v += kThreads) {
+      const int r = __ldcg(w.label + v);
+      cnt += (r >= 0 && (int)(uint32_t)__ldcg(w.ckey + r) == (int)v);
+    }
+    cnt = block_reduce_sum<int32_t>(cnt, sh.wtmp32);
+    if (threadIdx.x == 0) w.hist[blockIdx.x] = cnt;
+  }
+  grid_barrier(kp);
+  if (blockIdx.x == 0) {
+    const int x = threadIdx.x < kp.nblocks ? __ldcg(w.hist + threadIdx.x) : 0;
+    int tot;
+    const int ex = block_exclusive_scan<int32_t>(x, sh.wtmp32, tot);
+    if (threadIdx.x < kp.nblocks) w.hist[kp.nblocks + threadIdx.x] = ex;
+    if (threadIdx.x == 0) { w.sctl[0] = tot; w.sctl[1] = 0; }
+  }
+  grid_barrier(kp);
+  {
+    int run = __ldcg(w.hist + kp.nblocks + blockIdx.x);
+    for (long long base = cb; base < ce; base += kThreads) {
+      const long long v = base + threadIdx.x;
+      int r = -1, f = 0;
+      unsigned long long k = 0;
+      if (v < ce) {
+        r = __ldcg(w.label + v);
+        if (r >= 0) { k = __ldcg(w.ckey + r); f = (int)(uint32_t)k == (int)v; }
+      }
+      int tot;
+      const int ex = block_exclusive_scan<int32_t>(f, sh.wtmp32, tot);
+      if (f) {
+        w.keys0[run + ex] = ((k >> 32) << a.idbits) | (k & 0xffffffffull);
+        w.vals0[run + ex] = r;
+      }
+      run += tot;
+    }
   }
   grid_barrier(kp);
   stamp(kp, 5);
   int maxdeg = ld_cg_s32(&kp.ctl->maxdeg);
   int dbits = 0;
   while (dbits < 32 && (1ll << dbits) <= maxdeg) ++dbits;
-  radix_sort_phase(kp, w, a.idbits + dbits, reinterpret_cast<int32_t*>(sm.cand), sh);
+  radix_sort_phase(kp, w, a.idbits, a.idbits + dbits, reinterpret_cast<int32_t*>(sm.cand), sh);
   // offsets: exclusive scan of sizes in key order, after the chain-first total
   const int count = ld_cg_s32(w.sctl);
   const int cur = ld_cg_s32(w.sctl + 1);
   const int32_t* vals = cur ? w.vals1 : w.vals0;
-  if (blockIdx.x == 0) {
-    long long carry = ld_cg_s32(&kp.ctl->chain_total);
-    const int per = (count + kThreads - 1) / kThreads;
-    const int b0 = threadIdx.x * per, e0 = min(count, b0 + per);
+  chunk_of(kp, count, cb, ce);
+  {
     long long s = 0;
-    for (int i = b0; i < e0; ++i) s += __ldcg(w.csize + __ldcg(vals + i));
+    for (long long i = cb + threadIdx.x; i < ce; i += kThreads) s += __ldcg(w.csize + __ldcg(vals + i));
+    s = block_reduce_sum<long long>(s, sh.wtmpll);
+    if (threadIdx.x == 0) w.offs[blockIdx.x] = s;   // offs[] as per-block scratch first
+  }
+  grid_barrier(kp);
+  if (blockIdx.x == 0) {
+    const long long x = threadIdx.x < kp.nblocks ? __ldcg(w.offs + threadIdx.x) : 0;
     long long tot;
-    long long run = carry + block_exclusive_scan<long long>(s, sh.wtmpll, tot);
-    for (int i = b0; i < e0; ++i) { w.offs[i] = run; run += __ldcg(w.csize + __ldcg(vals + i)); }
+    const long long ex = block_exclusive_scan<long long>(x, sh.wtmpll, tot);
+    if (threadIdx.x < kp.nblocks) w.hist[threadIdx.x] = (int)ex;   // block bases (counts < 2^31)
     if (threadIdx.x == 0) {
       kp.ctl->n_comp = count;
       kp.ctl->n_chain = 0;
@@ -245,28 +347,37 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   Problem* chains = const_cast<Problem*>(kp.chains);
   Problem* solos = const_cast<Problem*>(kp.solos);
   int singles = 0;
-  for (int i = gtid(); i < count; i += G) {
-    const int root = __ldcg(vals + i);
-    const int size = __ldcg(w.csize + root);
-    const int seed = (int)(uint32_t)__ldcg(w.ckey + root);
-    const int pos = (int)__ldcg(w.offs + i);
-    if (size == 1) {
-      kp.o[pos] = seed;
-      kp.perm[n - 1 - pos] = seed;
-      if (kp.iperm) kp.iperm[seed] = n - 1 - pos;
-      ++singles;
-      continue;
-    }
-    Problem P;
-    P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
-    P.mat_n = n; P.pos0 = pos; P.size = size; P.seed = seed; P.pad = 0;
-    P.flags = a.mode == RCM_START_PSEUDO_PERIPHERAL ? 2 : 0;
-    if (a.thr > 0 && size <= a.thr) {
-      const int j = atomicAdd(&kp.ctl->n_solo, 1);
-      if (j < a.prob_cap) solos[j] = P; else latch_error(kp.ctl, ST_CAPACITY);
-    } else {
-      const int j = atomicAdd(&kp.ctl->n_chain, 1);
-      if (j < a.prob_cap) chains[j] = P; else latch_error(kp.ctl, ST_CAPACITY);
+  {
+    long long run = (long long)ld_cg_s32(&kp.ctl->chain_total) + __ldcg(w.hist + blockIdx.x);
+    for (long long base = cb; base < ce; base += kThreads) {
+      const long long i = base + threadIdx.x;
+      int root = -1, size = 0;
+      if (i < ce) { root = __ldcg(vals + i); size = __ldcg(w.csize + root); }
+      long long tot;
+      const long long ex = block_exclusive_scan<long long>((long long)size, sh.wtmpll, tot);
+      if (i < ce) {
+        const int seed = (int)(uint32_t)__ldcg(w.ckey + root);
+        const int pos = (int)(run + ex);
+        if (size == 1) {
+          kp.o[pos] = seed;
+          kp.perm[n - 1 - pos] = seed;
+          if (kp.iperm) kp.iperm[seed] = n - 1 - pos;
+          ++singles;
+        } else {
+          Problem P;
+          P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
+          P.mat_n = n; P.pos0 = pos; P.size = size; P.seed = seed; P.pad = 0;
+          P.flags = a.mode == RCM_START_PSEUDO_PERIPHERAL ? 2 : 0;
+          if (a.thr > 0 && size <= a.thr) {
+            const int j = atomicAdd(&kp.ctl->n_solo, 1);
+            if (j < a.prob_cap) solos[j] = P; else latch_error(kp.ctl, ST_CAPACITY);
+          } else {
+            const int j = atomicAdd(&kp.ctl->n_chain, 1);
+            if (j < a.prob_cap) chains[j] = P; else latch_error(kp.ctl, ST_CAPACITY);
+          }
+        }
+      }
+      run += tot;
     }
   }
   if (kp.collect_stats) {
