@@ -44,14 +44,23 @@ class rcm_options_t(ctypes.Structure):
                 ("solo_threshold", ctypes.c_int32), ("flags", ctypes.c_int32)]
 
 
+STAGES = ("dequeue", "parents", "discover", "wait_discovered", "rediscover_count", "sort",
+          "wait_counted", "output", "generate", "other")
+
+
 class rcm_stats_t(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "batches_generated", "batches_dequeued", "batches_executed", "batches_empty",
         "rediscover_early", "rediscover_late", "candidates_speculative", "candidates_removed",
-        "oversize_batches", "components", "overhang_forwards", "solo_problems")]
+        "oversize_batches", "components", "overhang_forwards", "solo_problems")] + [
+        ("stage_cycles", ctypes.c_int64 * 10)]
 
     def as_dict(self):
-        return {n: int(getattr(self, n)) for n, _ in self._fields_}
+        d = {n: int(getattr(self, n)) for n, _ in self._fields_ if n != "stage_cycles"}
+        cyc = [int(x) for x in self.stage_cycles]
+        if any(cyc):
+            d["stage_cycles"] = dict(zip(STAGES, cyc))
+        return d
 
 
 class RCMError(RuntimeError):

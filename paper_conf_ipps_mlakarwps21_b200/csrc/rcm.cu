@@ -144,11 +144,14 @@ __device__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemP
   }
   const int nsolo = ld_cg_s32(&kp.ctl->n_solo);
   for (;;) {
-    if (threadIdx.x == 0) sh.k = atomicAdd(&kp.ctl->solo_next, 1);
+    if (threadIdx.x == 0) {
+      sh.k = atomicAdd(&kp.ctl->solo_next, 1);
+      if (ld_cg_s32(&kp.ctl->status)) sh.k = nsolo;   // block-uniform exit decision
+    }
     __syncthreads();
     const int k = sh.k;
     __syncthreads();
-    if (k >= nsolo || ld_cg_s32(&kp.ctl->status)) break;
+    if (k >= nsolo) break;
     Problem P = kp.solos[k];
     if (P.size > 0) run_solo(kp, P, sm, sh, a.w.lev);
   }
@@ -265,6 +268,7 @@ struct rcm_plan {
   Problem* solos = nullptr;
   unsigned long long* pm_key = nullptr;
   unsigned long long* spill = nullptr;
+  int32_t* dbg = nullptr;
   CompWS w{};
 };
 
@@ -298,7 +302,7 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
                   p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
@@ -377,6 +381,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   AL(p->solos, sizeof(Problem) * p->prob_cap);
   AL(p->pm_key, 8 * p->prob_cap);
   AL(p->spill, 8 * 2 * p->spill_cap);
+  AL(p->dbg, 4 * 8 * 1024);
   AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
   AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
   AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kThreads)); AL(p->w.sctl, 4 * 64);
@@ -388,6 +393,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   if (cudaMemset(p->desc, 0, sizeof(Desc) * p->qcap) != cudaSuccess ||
       cudaMemset(p->sig, 0, sizeof(Sig) * (p->qcap + 1)) != cudaSuccess ||
       cudaMemset(p->ctl, 0, sizeof(Ctl)) != cudaSuccess || cudaMemset(p->stats, 0, sizeof(Stats)) != cudaSuccess ||
+      cudaMemset(p->dbg, 0, 4 * 8 * 1024) != cudaSuccess ||
       cudaDeviceSynchronize() != cudaSuccess) {
     st = RCM_ERR_CUDA;
     goto fail;
@@ -422,6 +428,7 @@ static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* 
   kp.flags = p->opt.flags;
   kp.collect_stats = p->opt.collect_stats;
   kp.nblocks = p->nblocks;
+  kp.dbg = p->dbg;
   return kp;
 }
 
@@ -538,6 +545,7 @@ extern "C" rcm_status_t rcm_get_stats(rcm_plan_t p, rcm_stats_t* out) {
   out->components = (int64_t)s.components;
   out->overhang_forwards = (int64_t)s.ovh_forwards;
   out->solo_problems = (int64_t)s.solo_problems;
+  for (int i = 0; i < 10; ++i) out->stage_cycles[i] = (int64_t)s.stage[i];
   return RCM_OK;
 }
 
@@ -566,6 +574,48 @@ extern "C" rcm_status_t rcm_debug_info(rcm_plan_t p, long long* out8) {
   if (!p || !out8) return RCM_ERR_INVALID_ARGUMENT;
   CK(cudaMemcpy(out8, p->ctl->dbg, 8 * sizeof(long long), cudaMemcpyDeviceToHost));
   return RCM_OK;
+}
+
+// Per-block progress beacons (nblocks x 8 int32: phase, slot, aux, count,
+// look-back j, word, iterations), copied on a private non-blocking stream so
+// it can be read while a launch is still running.  Not in the public header.
+extern "C" rcm_status_t rcm_debug_state(rcm_plan_t p, int32_t* host_out, int32_t* nblocks) {
+  if (!p || !host_out) return RCM_ERR_INVALID_ARGUMENT;
+  cudaStream_t s;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  cudaError_t e = cudaMemcpyAsync(host_out, p->dbg, 4 * 8 * p->nblocks, cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  if (nblocks) *nblocks = p->nblocks;
+  return e == cudaSuccess ? RCM_OK : RCM_ERR_CUDA;
+}
+
+// Raw chain slot state (desc + both status words) for slots [lo, lo+cnt):
+// 6 int64 per slot.  Debug only; copied on a private stream.
+extern "C" rcm_status_t rcm_debug_slots(rcm_plan_t p, int32_t lo, int32_t cnt, long long* host_out) {
+  if (!p || !host_out || lo < 0 || cnt <= 0 || lo + cnt > p->qcap) return RCM_ERR_INVALID_ARGUMENT;
+  cudaStream_t s;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  Sig* sg = (Sig*)malloc(sizeof(Sig) * cnt);
+  Desc* dd = (Desc*)malloc(sizeof(Desc) * cnt);
+  cudaMemcpyAsync(sg, p->sig + lo, sizeof(Sig) * cnt, cudaMemcpyDeviceToHost, s);
+  cudaMemcpyAsync(dd, p->desc + lo, sizeof(Desc) * cnt, cudaMemcpyDeviceToHost, s);
+  Ctl c;
+  cudaMemcpyAsync(&c, p->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s);
+  cudaError_t e = cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  for (int i = 0; i < cnt; ++i) {
+    host_out[6 * i + 0] = (long long)sg[i].word;
+    host_out[6 * i + 1] = (long long)sg[i].ovh;
+    host_out[6 * i + 2] = dd[i].o_begin;
+    host_out[6 * i + 3] = dd[i].o_end;
+    host_out[6 * i + 4] = dd[i].next;
+    host_out[6 * i + 5] = dd[i].tag;
+  }
+  host_out[6 * cnt] = c.head; host_out[6 * cnt + 1] = c.done; host_out[6 * cnt + 2] = c.qtail;
+  host_out[6 * cnt + 3] = c.completed; host_out[6 * cnt + 4] = c.epoch; host_out[6 * cnt + 5] = c.status;
+  free(sg); free(dd);
+  return e == cudaSuccess ? RCM_OK : RCM_ERR_CUDA;
 }
 
 extern "C" rcm_status_t rcm_plan_info(rcm_plan_t p, int64_t* out6) {

@@ -29,7 +29,20 @@ struct KParams {
   int32_t flags;
   int32_t collect_stats;
   int32_t nblocks;
+  int32_t* dbg;               // per-block progress (8 ints per block), always written
 };
+
+// Per-block progress beacon: phase, slot, aux -- polled by the host while the
+// kernel runs (rcm_debug_state) to diagnose stalls.  Thread 0 only.
+__device__ __forceinline__ void beacon(const KParams& kp, int phase, int slot, int aux) {
+  if (threadIdx.x == 0) {
+    volatile int32_t* d = kp.dbg + blockIdx.x * 8;
+    d[0] = phase;
+    d[1] = slot;
+    d[2] = aux;
+    d[3] = d[3] + 1;
+  }
+}
 
 enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16 };
 
@@ -84,7 +97,18 @@ struct ShState {
   unsigned long long minkey;
   int64_t spill_base;
   int32_t big_list[256];
+  long long clk[10];           // per-stage cycle accumulators (thread 0)
+  long long tclk;
 };
+
+// Stage clock: attribute the cycles since the last mark to stage i (thread 0).
+__device__ __forceinline__ void clk_mark(const KParams& kp, ShState& sh, int i) {
+  if (kp.collect_stats == 2 && threadIdx.x == 0) {
+    const long long now = clock64();
+    sh.clk[i] += now - sh.tclk;
+    sh.tclk = now;
+  }
+}
 
 __device__ __forceinline__ void latch_error(Ctl* ctl, int32_t code) {
   atomicCAS(&ctl->status, 0, code);

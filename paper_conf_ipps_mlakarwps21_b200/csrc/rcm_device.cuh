@@ -92,6 +92,11 @@ struct Ctl {
 struct Stats {
   unsigned long long generated, dequeued, executed, empty, redisc_early, redisc_late,
       cand_spec, cand_removed, oversize, components, ovh_forwards, solo_problems;
+  // per-stage SM cycles summed over workers (collect_stats == 2), the GPU
+  // analogue of the paper's Fig. 6 stage breakdown:
+  // dequeue, parents, discover, wait-Discovered, rediscover+count, sort,
+  // wait-Counted (prefix), output, generate, other
+  unsigned long long stage[10];
 };
 
 // ----------------------------------------------------------------- memory ops

@@ -59,18 +59,23 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
       continue;
     }
     j -= __ffs(~loc & need) - 1;   // verified-LOCAL slots stay LOCAL (monotone)
+    if (lane == 0 && (it & 63) == 63) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[4] = j; d[5] = (int)a; d[6] = it; }
     if (try_only && it >= 2) { *ready = 0; return true; }
     // A batch still waiting for Discovered has no aggregate yet, so it is a
     // successor of the batch that completed the order (which saw every
     // predecessor's aggregate): after early termination it has nothing to
     // output and may be abandoned -- and must be, since a slot it waits on may
     // have been abandoned at dequeue.
-    if (ld_relaxed_s32(&kp.ctl->status) || ld_relaxed_s32(&kp.ctl->done)) return false;
-    lb_spin(ns, it);
-    if ((it & 1023) == 1023) {
+    // every exit decision is taken warp-uniformly (lane 0's view, broadcast):
+    // lanes that left the loop on their own would strand the others in the
+    // full-mask ballots above
+    int quit = lane == 0 && (ld_relaxed_s32(&kp.ctl->status) || ld_relaxed_s32(&kp.ctl->done));
+    if ((it & 1023) == 1023 && lane == 0) {
       if (t0 == 0) t0 = globaltimer();
-      else if (globaltimer() - t0 > kWatchdogNs) { if (lane == 0) latch_hang(kp.ctl, 2, t, j, (long long)a); return false; }
+      else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 2, t, j, (long long)a); quit = 1; }
     }
+    if (__shfl_sync(0xffffffffu, quit, 0)) return false;
+    lb_spin(ns, it);
   }
   *ready = 1;
   return true;
@@ -85,6 +90,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
   unsigned ns = 0;
   uint64_t t0 = 0;
   for (int it = 0; j >= 0; ++it) {
+    if (lane == 0) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[4] = j; d[6] = it; d[7] = ld_relaxed_s32(&kp.ctl->done); }
     const int idx = j - lane;
     const bool valid = idx >= 0;
     const unsigned long long b = valid ? ld_acquire_u64(&kp.sig[idx].ovh) : 0ull;
@@ -121,12 +127,13 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
     // after early termination only batches without output may give up (a batch
     // with output precedes the terminating batch, whose look-back saw all of
     // its predecessors' aggregates, so this loop finishes)
-    if (ld_relaxed_s32(&kp.ctl->status) || (count == 0 && ld_relaxed_s32(&kp.ctl->done))) return false;
-    lb_spin(ns, it);
-    if ((it & 1023) == 1023) {
+    int quit = lane == 0 && (ld_relaxed_s32(&kp.ctl->status) || (count == 0 && ld_relaxed_s32(&kp.ctl->done)));
+    if ((it & 1023) == 1023 && lane == 0) {
       if (t0 == 0) t0 = globaltimer();
-      else if (globaltimer() - t0 > kWatchdogNs) { if (lane == 0) latch_hang(kp.ctl, 3, t, j, (long long)a); return false; }
+      else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 3, t, j, (long long)a); quit = 1; }
     }
+    if (__shfl_sync(0xffffffffu, quit, 0)) return false;   // warp-uniform exit
+    lb_spin(ns, it);
   }
   out_off = (int)(base_out + sc);
   q_off = (int)(base_q + sn);
@@ -145,17 +152,22 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
                          uint32_t epoch) {
   const int t = sh.t, o_begin = sh.o_begin;
   Sig* mine = kp.sig + t;
+  clk_mark(kp, sh, 0);
+  beacon(kp, 2, t, 0);
   const int nP = load_parents(kp, P, sm, sh, o_begin, sh.o_end - o_begin, false);
   const int E = sh.E;
   const bool oversize = E > kp.T;
   const uint32_t key0 = (uint32_t)o_begin + 1;
   if (threadIdx.x == 0) { sh.steal = 0; sh.aborted = 0; sh.s_early = 0; }
   __syncthreads();
+  clk_mark(kp, sh, 1);
   if (oversize) {
     if (!oversize_discover(kp, P, sm, sh, key0, sm.p_rs[0], E)) return;
   } else {
     discover(kp, P, sm, sh, o_begin, nP, E);
   }
+  clk_mark(kp, sh, 2);
+  beacon(kp, 4, t, 0);
   if (threadIdx.x == 0) {                       // own discovery done: LOCAL
     __threadfence();                            // the block's atomicMin marks first
     st_release_u64(&mine->word, LB_LOCAL);
@@ -167,6 +179,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     if (threadIdx.x == 0) { sh.s_early = ready; if (ready < 0) sh.aborted = 1; }
   }
   __syncthreads();
+  clk_mark(kp, sh, 3);
   if (sh.aborted) return;
   const bool early = sh.s_early == 1;
   if (early) {
@@ -178,14 +191,19 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
       st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));   // early Counted
       stat_add(kp, &kp.stats->redisc_early, 1);
     }
+    clk_mark(kp, sh, 4);
     if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
+    clk_mark(kp, sh, 5);
   } else {
     if (!oversize && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // speculative sort
+    clk_mark(kp, sh, 5);
+    beacon(kp, 6, t, 0);
     if (threadIdx.x < 32) {
       int ready = 0;
       if (!lb_wait_discovered(kp, t, false, &ready) && threadIdx.x == 0) sh.aborted = 1;
     }
     __syncthreads();
+    clk_mark(kp, sh, 3);
     if (sh.aborted) return;
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     if (oversize) {
@@ -200,11 +218,14 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
       st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));
       stat_add(kp, &kp.stats->redisc_late, 1);
     }
+    clk_mark(kp, sh, 4);
   }
   // Counted: prefix over the predecessors' aggregates
+  beacon(kp, 8, t, sh.count);
   if (threadIdx.x < 32) {
     int out_off = 0, q_off = 0;
     const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off);
+    if (threadIdx.x == 0) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[5] = 1000 + (int)ok; }
     if (threadIdx.x == 0) {
       if (!ok) {
         sh.aborted = 1;
@@ -220,8 +241,10 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     }
   }
   __syncthreads();
+  clk_mark(kp, sh, 6);
   if (sh.aborted) return;
   const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
+  beacon(kp, 9, t, out_off);
   GenState g;
   if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; }
   if (oversize) {
@@ -233,6 +256,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     write_output(kp, P, sm, sh, nP, E, out_off);
     __threadfence();
     __syncthreads();
+    clk_mark(kp, sh, 7);
     if (nb > 0) {
       build_prefix(kp, sm, sh, E);
       if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
@@ -274,10 +298,15 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     }
   }
   __syncthreads();
+  clk_mark(kp, sh, 8);
 }
 
 __device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                              uint32_t epoch) {
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 10; ++i) sh.clk[i] = 0;
+    sh.tclk = clock64();
+  }
   for (;;) {
     if (threadIdx.x == 0) sh.aborted = dequeue(kp, sh, epoch) ? 0 : 1;
     __syncthreads();
@@ -285,6 +314,10 @@ __device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs
     if (kp.flags & F_SERIAL_CHAIN) chain_batch(kp, P, sm, sh, epoch);   // Alg. 5 hand-off chain
     else lb_batch(kp, P, sm, sh, epoch);                                 // look-back chain
   }
+  clk_mark(kp, sh, 0);
+  beacon(kp, 12, -1, 0);
+  if (kp.collect_stats == 2 && threadIdx.x == 0)
+    for (int i = 0; i < 10; ++i) atomicAdd(&kp.stats->stage[i], (unsigned long long)sh.clk[i]);
   __syncthreads();
 }
 

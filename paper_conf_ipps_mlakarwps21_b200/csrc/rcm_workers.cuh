@@ -23,6 +23,7 @@ __device__ void place_root(const KParams& kp, const Problem& P, int s, int pos) 
 }
 
 __device__ void grid_barrier(const KParams& kp) {
+  beacon(kp, 11, -1, ld_relaxed_s32(&kp.ctl->gbar_gen));
   __syncthreads();
   if (threadIdx.x == 0) {
     int gen = ld_acquire_s32(&kp.ctl->gbar_gen);
@@ -356,6 +357,7 @@ __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
   for (;;) {
     if (ld_relaxed_s32(&kp.ctl->done)) return false;
     const int t = atomicAdd(&kp.ctl->head, 1);
+    beacon(kp, 1, t, 0);
     if (t >= kp.qcap) {   // only possible after a capacity error; wait for done
       while (!ld_relaxed_s32(&kp.ctl->done)) __nanosleep(1000);
       return false;

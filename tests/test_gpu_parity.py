@@ -182,3 +182,26 @@ def test_host_argument_errors(rcm):
     with pytest.raises(rcm.RCMError):
         rcm.rcm_reorder(plan.handle, 6, 8, rp, ci, oracle.FIXED, 0, perm)      # n above plan
     plan.close()
+
+
+@pytest.mark.parametrize("opts", [dict(), dict(batch_nodes=64), dict(flags=16)])
+def test_stress_no_stall_and_determinism(rcm, opts):
+    """Repeated runs on one plan: early termination races (a worker abandoning an
+    unpublished slot while others are mid look-back) must never stall; every
+    run must be bit-identical."""
+    import time
+    g, mode, start = synth.config_graph(2, "small")
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    plan = rcm.Plan(g.n, g.nnz, solo_threshold=-1, **opts)
+    rp, ci = _dev(g)
+    perm = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    t0 = time.time()
+    for _ in range(300):
+        rcm.rcm_reorder(plan.handle, g.n, g.nnz, rp, ci, mode, start, perm)
+    assert rcm.rcm_sync_status(plan.handle) == 0
+    assert time.time() - t0 < 60
+    assert np.array_equal(perm.cpu().numpy(), ref)
+    for _ in range(20):
+        plan.reorder(rp, ci, mode, start, perm=perm)
+        assert np.array_equal(perm.cpu().numpy(), ref)
+    plan.close()

@@ -27,13 +27,15 @@ def main():
         st = rcm.rcm_sync_status(plan.handle)
         ok = np.array_equal(perm.cpu().numpy(), ref)
         ph = plan.timing(); info = plan.info(); plan.close()
-        sp = rcm.Plan(g.n, g.nnz, collect_stats=1, **opts); sp.reorder(rp, ci, mode, start); stt = sp.stats(); sp.close()
+        sp = rcm.Plan(g.n, g.nnz, collect_stats=2, **opts); sp.reorder(rp, ci, mode, start); stt = sp.stats(); sp.close()
+        cyc = stt.get("stage_cycles", {}); tot = max(1, sum(cyc.values()))
         print(json.dumps({"cfg": cfg, "opts": opts, "ms_med": round(float(np.median(ts)), 4), "ms_min": round(min(ts), 4),
                           "ok": ok, "status": st, "phases": {k: round(v, 3) for k, v in ph.items()},
                           "T": info["temp_elems"], "blocks": info["blocks"],
                           "exec": stt["batches_executed"], "empty": stt["batches_empty"], "fwd": stt["overhang_forwards"],
                           "late": stt["rediscover_late"], "early": stt["rediscover_early"],
                           "removed": stt["candidates_removed"], "spec": stt["candidates_speculative"],
-                          "oversize": stt["oversize_batches"], "solo": stt["solo_problems"], "comps": stt["components"]}), flush=True)
+                          "oversize": stt["oversize_batches"], "solo": stt["solo_problems"], "comps": stt["components"],
+                          "stage_pct": {k: round(100 * v / tot, 1) for k, v in cyc.items()}}), flush=True)
 
 main()
