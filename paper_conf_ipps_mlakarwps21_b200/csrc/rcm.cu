@@ -125,7 +125,7 @@ __device__ void prologue_batched_phase(const KParams& kp, const MainArgs& a) {
 
 // The scheduling phase: every chain problem in turn on all blocks (grid
 // barrier between chains), then the solo problems, one per block at a time.
-__device__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
+__device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
   const int nchain = ld_cg_s32(&kp.ctl->n_chain);
   for (int c = 0; c < nchain; ++c) {
     if (kp.chains[c].flags & 2) {   // PSEUDO_PERIPHERAL component: GL seed first (C-5)
@@ -159,7 +159,8 @@ __device__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemP
 
 // One launch per call: reset -> prologue -> seed / problem set-up ->
 // traversal -> (components -> traversal).  Grid barriers between phases.
-__global__ void __launch_bounds__(kThreads, 2) k_main(KParams kp, MainArgs a) {
+template <int kMinBlocks>
+__global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(KParams kp, MainArgs a) {
   extern __shared__ __align__(16) unsigned char dsm[];
   __shared__ ShState sh;
   SmemPtrs sm = carve_smem(dsm, kp.BS, kp.T);
@@ -269,6 +270,7 @@ struct rcm_plan {
   unsigned long long* pm_key = nullptr;
   unsigned long long* spill = nullptr;
   int32_t* dbg = nullptr;
+  const void* kernel = nullptr;
   CompWS w{};
 };
 
@@ -335,7 +337,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
-  p->BS = o.batch_nodes ? o.batch_nodes : 512;
+  p->BS = o.batch_nodes ? o.batch_nodes : 256;
   const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
   const size_t static_sh = sizeof(ShState) + 64;
   // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per block)
@@ -349,12 +351,14 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   }
   p->T = T;
   p->smem = smem_bytes(p->BS, T);
-  if (cudaFuncSetAttribute(k_main, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
+  // one block per SM: the 128-register build (no spills); more: the 64-register build
+  p->kernel = bps == 1 ? (const void*)k_main<1> : (const void*)k_main<2>;
+  if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
     delete p;
     return RCM_ERR_CUDA;
   }
   int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_main, kThreads, p->smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, p->kernel, kThreads, p->smem);
   if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
   p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
   if (p->nblocks > kThreads) p->nblocks = kThreads / p->num_sms * p->num_sms;   // block-0 scans assume <= kThreads
@@ -454,7 +458,7 @@ static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& 
   KParams kpc = kp;
   MainArgs ac = a;
   void* args[] = {&kpc, &ac};
-  CK(cudaLaunchCooperativeKernel((const void*)k_main, dim3(p->nblocks), dim3(kThreads), args, p->smem, s));
+  CK(cudaLaunchCooperativeKernel(p->kernel, dim3(p->nblocks), dim3(kThreads), args, p->smem, s));
   return RCM_OK;
 }
 
