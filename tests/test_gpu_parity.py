@@ -205,3 +205,48 @@ def test_stress_no_stall_and_determinism(rcm, opts):
         plan.reorder(rp, ci, mode, start, perm=perm)
         assert np.array_equal(perm.cpu().numpy(), ref)
     plan.close()
+
+
+def test_c5_device_generator_matches_numpy(rcm):
+    import synth.device as sd
+    mats = [0, 1, 2, 3, 17, 4000]
+    b = sd.c5_generate(mats, num=8192)
+    sizes = synth.c5_sizes(8192)
+    rp = b["row_ptr_local"].cpu().numpy()
+    ci = b["col_idx_local"].cpu().numpy()
+    for i, k in enumerate(mats):
+        g = synth.c5_matrix(k, int(sizes[k]))
+        a, e = int(b["node_off_h"][i]), int(b["node_off_h"][i + 1])
+        assert np.array_equal(rp[a + i: e + i + 1], g.row_ptr)
+        assert np.array_equal(ci[int(b["nnz_off_h"][i]): int(b["nnz_off_h"][i + 1])], g.col_idx)
+    # and the batched traversal of the device-generated matrices
+    plan = rcm.Plan(b["total"], b["total_nnz"])
+    perm = plan.reorder_batched(b["node_off"], b["nnz_off"], b["row_ptr_local"], b["col_idx_local"],
+                                b["total"], b["total_nnz"]).cpu().numpy()
+    for i, k in enumerate(mats):
+        g = synth.c5_matrix(k, int(sizes[k]))
+        a, e = int(b["node_off_h"][i]), int(b["node_off_h"][i + 1])
+        assert np.array_equal(perm[a:e], oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE))
+    plan.close()
+
+
+def test_batched_pseudo_peripheral(rcm):
+    b = synth.c5_batch(num=12, seed=7, lo=30, hi=900)
+    ref = oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, oracle.PSEUDO_PERIPHERAL)
+    total, nnz = int(b.node_off[-1]), int(b.nnz_off[-1])
+    plan = rcm.Plan(total, nnz)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()  # noqa: E731
+    perm = plan.reorder_batched(t(b.node_off), t(b.nnz_off), t(b.row_ptr_local), t(b.col_idx_local),
+                                total, nnz, mode=oracle.PSEUDO_PERIPHERAL).cpu().numpy()
+    assert np.array_equal(perm, ref)
+    plan.close()
+
+
+def test_disconnected_pseudo_peripheral(rcm):
+    g = synth.disjoint_union([synth.grid2d(9, 7), synth.path(12), synth.star(5), synth.path(1),
+                              synth.relabel(synth.grid3d_27(5, 4, 6), synth.randperm(120, 3))])
+    g = synth.relabel(g, synth.randperm(g.n, 21))
+    ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.PSEUDO_PERIPHERAL, 0)
+    for opts in [dict(), dict(solo_threshold=-1, flags=8), dict(solo_threshold=8, flags=8)]:
+        got, _ = _run(rcm, g, oracle.PSEUDO_PERIPHERAL, 0, **opts)
+        assert np.array_equal(got, ref), opts
