@@ -270,6 +270,8 @@ struct rcm_plan {
   unsigned long long* pm_key = nullptr;
   unsigned long long* spill = nullptr;
   int32_t* dbg = nullptr;
+  unsigned long long* trace = nullptr;
+  int32_t trace_cap = 0;
   const void* kernel = nullptr;
   CompWS w{};
 };
@@ -304,7 +306,7 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
                   p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
@@ -386,6 +388,10 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   AL(p->pm_key, 8 * p->prob_cap);
   AL(p->spill, 8 * 2 * p->spill_cap);
   AL(p->dbg, 4 * 8 * 1024);
+  if (o.collect_stats == 3) {
+    p->trace_cap = (int32_t)std::min<int64_t>(p->qcap, 1 << 20);
+    AL(p->trace, 8 * 8 * (size_t)p->trace_cap);
+  }
   AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
   AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
   AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kThreads)); AL(p->w.sctl, 4 * 64);
@@ -433,6 +439,8 @@ static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* 
   kp.collect_stats = p->opt.collect_stats;
   kp.nblocks = p->nblocks;
   kp.dbg = p->dbg;
+  kp.trace = p->trace;
+  kp.trace_cap = p->trace_cap;
   return kp;
 }
 
@@ -455,6 +463,7 @@ static int bits_for(int64_t x) {
 // Cooperative launch: the runtime guarantees every block of the persistent
 // grid is co-resident (grid barriers and spin-waits rely on it) or fails.
 static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& a, cudaStream_t s) {
+  if (p->trace) CK(cudaMemsetAsync(p->trace, 0, 8 * 8 * (size_t)p->trace_cap, s));
   KParams kpc = kp;
   MainArgs ac = a;
   void* args[] = {&kpc, &ac};
@@ -592,6 +601,15 @@ extern "C" rcm_status_t rcm_debug_state(rcm_plan_t p, int32_t* host_out, int32_t
   cudaStreamDestroy(s);
   if (nblocks) *nblocks = p->nblocks;
   return e == cudaSuccess ? RCM_OK : RCM_ERR_CUDA;
+}
+
+// Per-slot event trace of the last call (collect_stats == 3): copies
+// min(cnt, trace_cap) * 8 u64.  Debug / analysis only.
+extern "C" rcm_status_t rcm_debug_trace(rcm_plan_t p, int32_t cnt, unsigned long long* host_out) {
+  if (!p || !host_out || !p->trace) return RCM_ERR_INVALID_ARGUMENT;
+  const int32_t c = std::min(cnt, p->trace_cap);
+  CK(cudaMemcpy(host_out, p->trace, 8 * 8 * (size_t)c, cudaMemcpyDeviceToHost));
+  return RCM_OK;
 }
 
 // Raw chain slot state (desc + both status words) for slots [lo, lo+cnt):

@@ -30,7 +30,21 @@ struct KParams {
   int32_t collect_stats;
   int32_t nblocks;
   int32_t* dbg;               // per-block progress (8 ints per block), always written
+  unsigned long long* trace;  // nullable: per-slot event times (collect_stats == 3)
+  int32_t trace_cap;          // slots traced
 };
+
+// Per-slot event trace (collect_stats == 3): %globaltimer at dequeue (0),
+// discovery done (1), Discovered known (2), aggregate published (3), prefix
+// known (4), output written (5), batches published (6); [7] = generator slot
+// << 32 | block.  Thread 0 only.
+__device__ __forceinline__ void trace_ev(const KParams& kp, int slot, int ev) {
+  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && slot >= 0 && slot < kp.trace_cap) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    kp.trace[(size_t)slot * 8 + ev] = t;
+  }
+}
 
 // Per-block progress beacon: phase, slot, aux -- polled by the host while the
 // kernel runs (rcm_debug_state) to diagnose stalls.  Thread 0 only.

@@ -6,7 +6,10 @@
 
 namespace rcm {
 
-constexpr int kThreads = 512;               // threads per persistent worker block
+#ifndef RCM_THREADS
+#define RCM_THREADS 512
+#endif
+constexpr int kThreads = RCM_THREADS;       // threads per persistent worker block
 constexpr int kWarps = kThreads / 32;
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner

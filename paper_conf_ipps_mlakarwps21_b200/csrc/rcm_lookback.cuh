@@ -168,6 +168,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   }
   clk_mark(kp, sh, 2);
   beacon(kp, 4, t, 0);
+  trace_ev(kp, t, 1);
   if (threadIdx.x == 0) {                       // own discovery done: LOCAL
     __threadfence();                            // the block's atomicMin marks first
     st_release_u64(&mine->word, LB_LOCAL);
@@ -183,6 +184,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   if (sh.aborted) return;
   const bool early = sh.s_early == 1;
   if (early) {
+    trace_ev(kp, t, 2);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     rediscover(kp, P, sm, sh, o_begin, E);      // dense array after sorting
     count_outputs(kp, sm, sh, nP, E);
@@ -205,6 +207,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     __syncthreads();
     clk_mark(kp, sh, 3);
     if (sh.aborted) return;
+    trace_ev(kp, t, 2);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     if (oversize) {
       oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
@@ -222,6 +225,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   }
   // Counted: prefix over the predecessors' aggregates
   beacon(kp, 8, t, sh.count);
+  trace_ev(kp, t, 3);
   if (threadIdx.x < 32) {
     int out_off = 0, q_off = 0;
     const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off);
@@ -245,6 +249,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   if (sh.aborted) return;
   const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
   beacon(kp, 9, t, out_off);
+  trace_ev(kp, t, 4);
   GenState g;
   if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; }
   if (oversize) {
@@ -257,6 +262,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     __threadfence();
     __syncthreads();
     clk_mark(kp, sh, 7);
+    trace_ev(kp, t, 5);
     if (nb > 0) {
       build_prefix(kp, sm, sh, E);
       if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
@@ -271,6 +277,10 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     stat_add(kp, &kp.stats->executed, 1);
   }
   __syncthreads();
+  trace_ev(kp, t, 6);
+  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
+    for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
+      kp.trace[(size_t)(q_off + i) * 8 + 7] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
   // empty slots: published as discovered with a zero aggregate
   const int emitted = sh.k;
   if (nb > emitted && threadIdx.x < 32) {

@@ -379,6 +379,7 @@ __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
     const int b = ld_relaxed_s32(&d->o_begin), e = ld_relaxed_s32(&d->o_end), nx = ld_relaxed_s32(&d->next);
     stat_add(kp, &kp.stats->dequeued, 1);
     if (b == e) { stat_add(kp, &kp.stats->empty, 1); continue; }
+    trace_ev(kp, t, 0);
     sh.t = t;
     sh.o_begin = b;
     sh.o_end = e;
