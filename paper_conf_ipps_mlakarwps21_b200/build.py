@@ -31,6 +31,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     extra = [f"-DRCM_THREADS={os.environ['RCM_THREADS']}"] if os.environ.get("RCM_THREADS") else []
+    if os.environ.get("RCM_TRACE"):
+        extra.append("-DRCM_TRACE")
     cmd = [NVCC, *FLAGS, *extra, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")

@@ -38,12 +38,19 @@ struct KParams {
 // discovery done (1), Discovered known (2), aggregate published (3), prefix
 // known (4), output written (5), batches published (6); [7] = generator slot
 // << 32 | block.  Thread 0 only.
-__device__ __forceinline__ void trace_ev(const KParams& kp, int slot, int ev) {
-  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && slot >= 0 && slot < kp.trace_cap) {
+__device__ __noinline__ void trace_ev_slow(unsigned long long* trace, int cap, int slot, int ev) {
+  if (trace && slot >= 0 && slot < cap) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    kp.trace[(size_t)slot * 8 + ev] = t;
+    trace[(size_t)slot * 8 + ev] = t;
   }
+}
+// Compiled in only with -DRCM_TRACE (the extra code changes the inlining and
+// register allocation of the persistent kernel).
+__device__ __forceinline__ void trace_ev(const KParams& kp, int slot, int ev) {
+#ifdef RCM_TRACE
+  if (kp.collect_stats == 3 && threadIdx.x == 0) trace_ev_slow(kp.trace, kp.trace_cap, slot, ev);
+#endif
 }
 
 // Per-block progress beacon: phase, slot, aux -- polled by the host while the

@@ -278,9 +278,11 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   }
   __syncthreads();
   trace_ev(kp, t, 6);
+#ifdef RCM_TRACE
   if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
     for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
       kp.trace[(size_t)(q_off + i) * 8 + 7] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
+#endif
   // empty slots: published as discovered with a zero aggregate
   const int emitted = sh.k;
   if (nb > emitted && threadIdx.x < 32) {
