@@ -24,6 +24,7 @@ RCM_FLAG_NO_EARLY = 0x2
 RCM_FLAG_NO_SORT = 0x4
 RCM_FLAG_FORCE_CHAIN = 0x8
 RCM_FLAG_SERIAL_CHAIN = 0x10
+RCM_FLAG_LEVELED = 0x20
 
 STATUS = {
     0: "RCM_OK", 1: "RCM_ERR_INVALID_ARGUMENT", 2: "RCM_ERR_BAD_CSR", 3: "RCM_ERR_NOT_SYMMETRIC",

@@ -9,7 +9,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librcm.so")
 SOURCES = ["rcm.cu"]
-HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh"]
+HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh", "rcm_leveled.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2", "-cudart", "static", "-shared",

@@ -11,6 +11,7 @@
 #include "../../include/rcm.h"
 #include "rcm_lookback.cuh"
 #include "rcm_components.cuh"
+#include "rcm_leveled.cuh"
 
 using namespace rcm;
 
@@ -132,6 +133,11 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
       const int x = gl_phase(kp, a.w, a.n, kp.chains[c].seed, sh);
       if (blockIdx.x == 0 && threadIdx.x == 0) const_cast<Problem*>(kp.chains)[c].seed = x;
       grid_barrier(kp);
+    }
+    if (kp.flags & F_LEVELED) {      // NEXT-3: Alg. 2 level-synchronous traversal
+      const Problem PL = kp.chains[c];
+      leveled_chain(kp, a, PL, sm, sh);
+      continue;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) chain_init(kp, kp.chains[c]);
     grid_barrier(kp);

@@ -65,7 +65,8 @@ __device__ __forceinline__ void beacon(const KParams& kp, int phase, int slot, i
   }
 }
 
-enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16 };
+enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16,
+                 F_LEVELED = 32 };
 
 // Dynamic shared memory of one worker.
 struct SmemPtrs {

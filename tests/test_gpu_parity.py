@@ -62,6 +62,7 @@ PATHS = {
     "serial": dict(flags=8 | 16, solo_threshold=-1),                 # Alg. 5 hand-off chain
     "serial_bs3_noovh": dict(flags=8 | 16 | 1, solo_threshold=-1, batch_nodes=3),
     "serial_noearly": dict(flags=8 | 16 | 2, solo_threshold=-1, batch_nodes=7, temp_elems=2304),
+    "leveled": dict(flags=8 | 32, solo_threshold=-1),                # Alg. 2 (NEXT-3)
 }
 
 
@@ -76,7 +77,7 @@ def test_tiny_families(rcm, path):
 
 
 @pytest.mark.parametrize("cfg", [1, 2, 3, 4])
-@pytest.mark.parametrize("path", ["solo", "chain", "serial", "serial_bs3_noovh"])
+@pytest.mark.parametrize("path", ["solo", "chain", "serial", "serial_bs3_noovh", "leveled"])
 def test_config_small_twins(rcm, cfg, path):
     g, mode, start = synth.config_graph(cfg, "small")
     ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
@@ -128,6 +129,15 @@ def test_full_config_parity(rcm, cfg):
     got, st = _run(rcm, g, mode, start, collect_stats=1)
     assert np.array_equal(got, ref)
     assert verify(g.row_ptr, g.col_idx, got, mode, start) is None
+
+
+@pytest.mark.parametrize("cfg", [1, 2, 3, 4])
+def test_full_config_parity_leveled(rcm, cfg):
+    """NEXT-3: Alg. 2 on the GPU -- a second, independent implementation."""
+    g, mode, start = synth.config_graph(cfg)
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    got, _ = _run(rcm, g, mode, start, flags=8 | 32, solo_threshold=-1)
+    assert np.array_equal(got, ref)
 
 
 @pytest.mark.parametrize("cfg", [3, 4])
