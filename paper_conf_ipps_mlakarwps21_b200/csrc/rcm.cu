@@ -441,6 +441,8 @@ static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* 
   kp.qcap = (int32_t)p->qcap;
   kp.BS = p->BS;
   kp.T = p->T;
+  kp.Bg = p->BS;
+  kp.Tg = p->T;
   kp.flags = p->opt.flags;
   kp.collect_stats = p->opt.collect_stats;
   kp.nblocks = p->nblocks;
@@ -485,6 +487,13 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
   if (mode == RCM_START_FIXED && (start < 0 || start >= n)) return RCM_ERR_INVALID_ARGUMENT;
   KParams kp = make_kparams(p, row_ptr, col_idx, perm, iperm);
+  if (!p->opt.batch_nodes && !p->opt.temp_elems && nnz >= 20ll * n) {
+    // dense rows (FEM-like, average valence >= 20): smaller batches shorten the
+    // critical generation chain; sparse graphs keep
+    // the shared-memory maxima
+    kp.Bg = std::min(kp.BS, 160);
+    kp.Tg = std::min(kp.T, 6144);
+  }
   MainArgs a = make_args(p);
   a.n = n;
   a.nnz = nnz;

@@ -24,8 +24,10 @@ struct KParams {
   unsigned long long* spill;  // oversize scratch: [0, spill_cap) keys, [spill_cap, 2*spill_cap) temp
   int64_t spill_cap;
   int32_t qcap;
-  int32_t BS;                 // B_s
-  int32_t T;                  // temp elements per batch
+  int32_t BS;                 // B_s capacity (shared-memory layout)
+  int32_t T;                  // temp-element capacity per batch (shared memory)
+  int32_t Bg;                 // B_s used to cut new batches (<= BS)
+  int32_t Tg;                 // valence budget used to cut new batches (<= T)
   int32_t flags;
   int32_t collect_stats;
   int32_t nblocks;
@@ -400,7 +402,7 @@ __device__ void count_outputs(const KParams& kp, const SmemPtrs& sm, ShState& sh
     unsigned long long k = sm.cand[e];
     if (k == kKeyMax) continue;
     long long d = (long long)(k >> 32);
-    v += d < kp.T ? d : kp.T;
+    v += d < kp.Tg ? d : kp.Tg;
   }
   long long V = block_reduce_sum<long long>(v, sh.wtmpll);
   int c = 0;
@@ -509,7 +511,7 @@ __device__ void gen_chunk(const KParams& kp, GenState& g, const unsigned long lo
       unsigned long long p = pre[mid];
       int c = (int)(p >> 40) - ca;
       long long v = (long long)((p & kMaskV) - (pa & kMaskV));
-      if (g.cnt + c <= kp.BS && g.val + v <= kp.T) lo = mid; else hi = mid - 1;
+      if (g.cnt + c <= kp.Bg && g.val + v <= kp.Tg) lo = mid; else hi = mid - 1;
     }
     int taken = (int)(pre[lo] >> 40) - ca;
     if (taken == 0) {
@@ -548,7 +550,7 @@ __device__ void build_prefix(const KParams& kp, const SmemPtrs& sm, ShState& sh,
     int lp = sm.lpof[i];
     if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
       unsigned long long d = sm.cand[i] >> 32;
-      s += (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+      s += (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
     }
   }
   unsigned long long tot;
@@ -558,7 +560,7 @@ __device__ void build_prefix(const KParams& kp, const SmemPtrs& sm, ShState& sh,
     unsigned long long x = 0;
     if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
       unsigned long long d = sm.cand[i] >> 32;
-      x = (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+      x = (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
     }
     sm.cand[i] = run;
     run += x;

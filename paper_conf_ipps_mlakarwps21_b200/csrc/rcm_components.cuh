@@ -12,7 +12,7 @@
 
 namespace rcm {
 
-constexpr int kSortTile = 4096;   // keys per tile of a radix pass (8 per thread)
+constexpr int kSortTile = 8 * kThreads;   // keys per tile of a radix pass (8 per thread)
 
 struct CompWS {
   int32_t* label;              // union-find parent (-1: already ordered)

@@ -11,6 +11,7 @@ namespace rcm {
 #endif
 constexpr int kThreads = RCM_THREADS;       // threads per persistent worker block
 constexpr int kWarps = kThreads / 32;
+static_assert(kThreads % 32 == 0 && kThreads >= 256 && kThreads <= 1024, "block size");
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner
 constexpr uint64_t kKeyMax = ~0ull;         // removed / padding sort key

@@ -143,8 +143,8 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
 __device__ __forceinline__ int lb_nb(const KParams& kp, int N, long long V) {
   if (N <= 0) return 0;
   // safe over-estimate of the greedy batch count
-  const long long v2 = (2 * V + kp.T - 1) / kp.T;
-  return N / kp.BS + (int)(v2 > 1 ? v2 : 1);
+  const long long v2 = (2 * V + kp.Tg - 1) / kp.Tg;
+  return N / kp.Bg + (int)(v2 > 1 ? v2 : 1);
 }
 
 // Process one dequeued batch with the look-back chain.

@@ -199,7 +199,7 @@ __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, c
       int c = __ldg(col + i * 32 + j);
       unsigned long long w = ld_relaxed_u64(word + c);
       if ((uint32_t)(w >> 32) != key) { keep &= ~(1u << j); ++removed; }
-      else { ++cnt; long long d = (long long)(w & 0xffffffffull); val += d < kp.T ? d : kp.T; }
+      else { ++cnt; long long d = (long long)(w & 0xffffffffull); val += d < kp.Tg ? d : kp.Tg; }
     }
     bits[i] = keep;
   }
@@ -282,14 +282,14 @@ __device__ void oversize_output(const KParams& kp, const Problem& P, const SmemP
     unsigned long long s = 0;
     for (int i = b; i < e; ++i) {
       unsigned long long d = __ldcg(src + c0 + i) >> 32;
-      s += (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+      s += (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
     }
     unsigned long long tot;
     unsigned long long run = block_exclusive_scan<unsigned long long>(s, sh.wtmp64, tot);
     for (int i = b; i < e; ++i) {
       unsigned long long d = __ldcg(src + c0 + i) >> 32;
       sm.cand[i] = run;
-      run += (1ull << 40) | (d < (unsigned long long)kp.T ? d : (unsigned long long)kp.T);
+      run += (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
     }
     if (threadIdx.x == 0) sm.cand[m] = tot;
     __syncthreads();
@@ -317,8 +317,8 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, un
   const long long Vp = (long long)ovh_t + sh.V;
   // combine with next: below half a batch in nodes and temp
   // elements, and a successor slot already exists (else nobody would receive it)
-  const bool fwd = !(kp.flags & F_NO_OVERHANG) && Np > 0 && 2 * Np < kp.BS &&
-                   2 * Vp < (long long)kp.T && succ < q_off;
+  const bool fwd = !(kp.flags & F_NO_OVERHANG) && Np > 0 && 2 * Np < kp.Bg &&
+                   2 * Vp < (long long)kp.Tg && succ < q_off;
   int nb = 0;
   if (fwd) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(&succ_sig->ovh),
@@ -329,8 +329,8 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, un
     if (Np > 0) {
       // safe over-estimate of the greedy batch count:
       // floor(N/B_s) + max(1, ceil(2V/T))  (P:L800-809 uses 2x the ideal count)
-      const long long v2 = (2 * Vp + kp.T - 1) / kp.T;
-      nb = Np / kp.BS + (int)(v2 > 1 ? v2 : 1);
+      const long long v2 = (2 * Vp + kp.Tg - 1) / kp.Tg;
+      nb = Np / kp.Bg + (int)(v2 > 1 ? v2 : 1);
     }
     if ((long long)q_off + nb > kp.qcap) {
       latch_error(kp.ctl, ST_CAPACITY);
