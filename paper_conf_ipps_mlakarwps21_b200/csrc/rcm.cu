@@ -353,6 +353,12 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
       std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
   int T = o.temp_elems;
   if (!T) T = (int)((per_block - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
+  if (!o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max) {
+    // dense rows (FEM-like): smaller batches shorten the critical generation
+    // chain, and the shared memory left over serves as L1
+    T = std::min(T, 6144);
+    p->BS = 160;
+  }
   if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;
@@ -488,9 +494,8 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   if (mode == RCM_START_FIXED && (start < 0 || start >= n)) return RCM_ERR_INVALID_ARGUMENT;
   KParams kp = make_kparams(p, row_ptr, col_idx, perm, iperm);
   if (!p->opt.batch_nodes && !p->opt.temp_elems && nnz >= 20ll * n) {
-    // dense rows (FEM-like, average valence >= 20): smaller batches shorten the
-    // critical generation chain; sparse graphs keep
-    // the shared-memory maxima
+    // dense rows (FEM-like, average valence >= 20) on a plan sized for sparser
+    // graphs: cut smaller batches
     kp.Bg = std::min(kp.BS, 160);
     kp.Tg = std::min(kp.T, 6144);
   }
