@@ -13,7 +13,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "librcm.so")
+# RCM_LIB: an alternative in-tree build of the same library (A/B experiments, tools/)
+LIB_PATH = os.environ.get("RCM_LIB") or os.path.join(_HERE, "librcm.so")
 
 RCM_START_FIXED = 0
 RCM_START_MIN_DEGREE = 1

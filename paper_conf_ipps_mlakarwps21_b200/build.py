@@ -31,6 +31,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     extra = [f"-DRCM_THREADS={os.environ['RCM_THREADS']}"] if os.environ.get("RCM_THREADS") else []
+    if os.environ.get("RCM_DISC_U"):
+        extra.append(f"-DRCM_DISC_U={os.environ['RCM_DISC_U']}")
     if os.environ.get("RCM_TRACE"):
         extra.append("-DRCM_TRACE")
     cmd = [NVCC, *FLAGS, *extra, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]

@@ -142,8 +142,11 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
     if (blockIdx.x == 0 && threadIdx.x == 0) chain_init(kp, kp.chains[c]);
     grid_barrier(kp);
     const uint32_t epoch = ld_acquire_u32(&kp.ctl->epoch);
-    const Problem P = kp.chains[c];
-    chain_worker(kp, P, sm, sh, epoch);
+    // the problem lives in shared memory: its fields are re-read on use (LDS)
+    // instead of pinning 16 registers across the whole traversal
+    if (threadIdx.x == 0) sh.prob = kp.chains[c];
+    __syncthreads();
+    chain_worker(kp, sh.prob, sm, sh, epoch);
     grid_barrier(kp);
     chain_reset_signals(kp);
     grid_barrier(kp);
@@ -158,17 +161,19 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
     const int k = sh.k;
     __syncthreads();
     if (k >= nsolo) break;
-    Problem P = kp.solos[k];
-    if (P.size > 0) run_solo(kp, P, sm, sh, a.w.lev);
+    if (threadIdx.x == 0) sh.prob = kp.solos[k];
+    __syncthreads();
+    if (sh.prob.size > 0) run_solo(kp, sh.prob, sm, sh, a.w.lev);
+    __syncthreads();
   }
 }
 
 // One launch per call: reset -> prologue -> seed / problem set-up ->
 // traversal -> (components -> traversal).  Grid barriers between phases.
 template <int kMinBlocks>
-__global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(KParams kp, MainArgs a) {
-  extern __shared__ __align__(16) unsigned char dsm[];
+__global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_constant__ KParams kp, const __grid_constant__ MainArgs a) {
   __shared__ ShState sh;
+  extern __shared__ __align__(16) unsigned char dsm[];
   SmemPtrs sm = carve_smem(dsm, kp.BS, kp.T);
   const int G = gthreads(kp);
   // ---- phase 0: reset the per-call control state
@@ -402,7 +407,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   AL(p->dbg, 4 * 8 * 1024);
   if (o.collect_stats == 3) {
     p->trace_cap = (int32_t)std::min<int64_t>(p->qcap, 1 << 20);
-    AL(p->trace, 8 * 8 * (size_t)p->trace_cap);
+    AL(p->trace, 8 * kTraceW * (size_t)p->trace_cap);
   }
   AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
   AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
@@ -477,7 +482,7 @@ static int bits_for(int64_t x) {
 // Cooperative launch: the runtime guarantees every block of the persistent
 // grid is co-resident (grid barriers and spin-waits rely on it) or fails.
 static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& a, cudaStream_t s) {
-  if (p->trace) CK(cudaMemsetAsync(p->trace, 0, 8 * 8 * (size_t)p->trace_cap, s));
+  if (p->trace) CK(cudaMemsetAsync(p->trace, 0, 8 * kTraceW * (size_t)p->trace_cap, s));
   KParams kpc = kp;
   MainArgs ac = a;
   void* args[] = {&kpc, &ac};
@@ -624,11 +629,11 @@ extern "C" rcm_status_t rcm_debug_state(rcm_plan_t p, int32_t* host_out, int32_t
 }
 
 // Per-slot event trace of the last call (collect_stats == 3): copies
-// min(cnt, trace_cap) * 8 u64.  Debug / analysis only.
+// min(cnt, trace_cap) * kTraceW u64.  Debug / analysis only.
 extern "C" rcm_status_t rcm_debug_trace(rcm_plan_t p, int32_t cnt, unsigned long long* host_out) {
   if (!p || !host_out || !p->trace) return RCM_ERR_INVALID_ARGUMENT;
   const int32_t c = std::min(cnt, p->trace_cap);
-  CK(cudaMemcpy(host_out, p->trace, 8 * 8 * (size_t)c, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(host_out, p->trace, 8 * kTraceW * (size_t)c, cudaMemcpyDeviceToHost));
   return RCM_OK;
 }
 

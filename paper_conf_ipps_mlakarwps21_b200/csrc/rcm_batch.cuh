@@ -36,15 +36,17 @@ struct KParams {
   int32_t trace_cap;          // slots traced
 };
 
-// Per-slot event trace (collect_stats == 3): %globaltimer at dequeue (0),
-// discovery done (1), Discovered known (2), aggregate published (3), prefix
-// known (4), output written (5), batches published (6); [7] = generator slot
-// << 32 | block.  Thread 0 only.
+// Per-slot event trace (collect_stats == 3), kTraceW words per slot:
+// %globaltimer at dequeue (0), parents loaded (1), discovery done (2),
+// Discovered known (3), aggregate published (4), before the prefix look-back
+// (5), prefix known (6), output written (7), batches published (8);
+// [kTraceW-1] = generator slot << 32 | block.  Thread 0 only.
+constexpr int kTraceW = 16;
 __device__ __noinline__ void trace_ev_slow(unsigned long long* trace, int cap, int slot, int ev) {
   if (trace && slot >= 0 && slot < cap) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    trace[(size_t)slot * 8 + ev] = t;
+    trace[(size_t)slot * kTraceW + ev] = t;
   }
 }
 // Compiled in only with -DRCM_TRACE (the extra code changes the inlining and
@@ -55,15 +57,17 @@ __device__ __forceinline__ void trace_ev(const KParams& kp, int slot, int ev) {
 #endif
 }
 
-// Per-block progress beacon: phase, slot, aux -- polled by the host while the
-// kernel runs (rcm_debug_state) to diagnose stalls.  Thread 0 only.
+// Per-block progress beacon: phase, slot, aux, SM clock -- polled by the host
+// while the kernel runs (rcm_debug_state) to diagnose stalls.  Thread 0 only.
+// Store-only: a read-modify-write here would put a memory round trip on the
+// block's critical path at every call.
 __device__ __forceinline__ void beacon(const KParams& kp, int phase, int slot, int aux) {
   if (threadIdx.x == 0) {
     volatile int32_t* d = kp.dbg + blockIdx.x * 8;
     d[0] = phase;
     d[1] = slot;
     d[2] = aux;
-    d[3] = d[3] + 1;
+    d[3] = (int32_t)clock();
   }
 }
 
@@ -123,6 +127,7 @@ struct ShState {
   int32_t big_list[256];
   long long clk[10];           // per-stage cycle accumulators (thread 0)
   long long tclk;
+  Problem prob;                // the problem being traversed (chain or solo)
 };
 
 // Stage clock: attribute the cycles since the last mark to stage i (thread 0).
@@ -471,8 +476,7 @@ __device__ __forceinline__ void publish_desc(Desc* d, int b, int e, int next, ui
   d->o_begin = b;
   d->o_end = e;
   d->next = next;
-  __threadfence();
-  st_release_u32(&d->tag, epoch);
+  st_release_u32(&d->tag, epoch);   // release: orders the fields above (and, cumulatively, what the block wrote before its last barrier)
 }
 
 __device__ __forceinline__ void gen_close(const KParams& kp, GenState& g, int end, int q_off,

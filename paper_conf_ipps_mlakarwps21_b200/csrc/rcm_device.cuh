@@ -12,6 +12,10 @@ namespace rcm {
 constexpr int kThreads = RCM_THREADS;       // threads per persistent worker block
 constexpr int kWarps = kThreads / 32;
 static_assert(kThreads % 32 == 0 && kThreads >= 256 && kThreads <= 1024, "block size");
+#ifndef RCM_DISC_U
+#define RCM_DISC_U 8
+#endif
+constexpr int kDiscU = RCM_DISC_U;          // edge slots per thread in flight in discovery
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner
 constexpr uint64_t kKeyMax = ~0ull;         // removed / padding sort key
@@ -129,8 +133,23 @@ __device__ __forceinline__ int32_t ld_relaxed_s32(const int32_t* p) {
   asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// Acquire side of a relaxed polling loop.  On sm_100a every ld.acquire.gpu is
+// an LDG.STRONG followed by CCTL.IVALL, which drops the whole SM's L1 (the
+// other resident block's cached lines and spill slots included), so spin
+// loops poll with relaxed loads and pay for one acquire fence after they exit
+// (PTX memory model: relaxed load observing a release + fence.acq_rel = acquire
+// pattern).
+__device__ __forceinline__ void fence_acquire_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 __device__ __forceinline__ void st_release_u64(unsigned long long* p, unsigned long long v) {
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void red_release_add_s32(int32_t* p, int32_t v) {
+  asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 __device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");

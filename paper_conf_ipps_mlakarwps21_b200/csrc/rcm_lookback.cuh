@@ -48,7 +48,7 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
   uint64_t t0 = 0;
   for (int it = 0; j >= 0; ++it) {
     const int idx = j - lane;
-    const unsigned long long a = idx >= 0 ? ld_acquire_u64(&kp.sig[idx].word) : (LB_LOCAL | LB_DINCL);
+    const unsigned long long a = idx >= 0 ? ld_relaxed_u64(&kp.sig[idx].word) : (LB_LOCAL | LB_DINCL);
     const unsigned incl = __ballot_sync(0xffffffffu, (a & LB_DINCL) != 0);
     const unsigned loc = __ballot_sync(0xffffffffu, (a & LB_LOCAL) != 0);
     const int stop = incl ? __ffs(incl) - 1 : 32;
@@ -77,6 +77,10 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
     if (__shfl_sync(0xffffffffu, quit, 0)) return false;
     lb_spin(ns, it);
   }
+  // the flags were polled relaxed: one acquire fence orders this block's
+  // rediscovery loads (after the caller's barrier) behind the predecessors'
+  // LOCAL/DINCL releases, i.e. behind their atomicMin marks
+  fence_acquire_gpu();
   *ready = 1;
   return true;
 }
@@ -90,11 +94,12 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
   unsigned ns = 0;
   uint64_t t0 = 0;
   for (int it = 0; j >= 0; ++it) {
-    if (lane == 0) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[4] = j; d[6] = it; d[7] = ld_relaxed_s32(&kp.ctl->done); }
+    if (lane == 0 && (it & 63) == 63) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[4] = j; d[6] = it; }
     const int idx = j - lane;
     const bool valid = idx >= 0;
-    const unsigned long long b = valid ? ld_acquire_u64(&kp.sig[idx].ovh) : 0ull;
-    const unsigned long long a = valid ? ld_acquire_u64(&kp.sig[idx].word) : 0ull;
+    // relaxed: the prefix needs only the values carried in the status words
+    const unsigned long long b = valid ? ld_relaxed_u64(&kp.sig[idx].ovh) : 0ull;
+    const unsigned long long a = valid ? ld_relaxed_u64(&kp.sig[idx].word) : 0ull;
     const unsigned incl = __ballot_sync(0xffffffffu, !valid || (b & 1ull));
     const unsigned agg = __ballot_sync(0xffffffffu, valid && (a & LB_AGG));
     const int stop = incl ? __ffs(incl) - 1 : 32;
@@ -148,13 +153,14 @@ __device__ __forceinline__ int lb_nb(const KParams& kp, int N, long long V) {
 }
 
 // Process one dequeued batch with the look-back chain.
-__device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+__device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                          uint32_t epoch) {
   const int t = sh.t, o_begin = sh.o_begin;
   Sig* mine = kp.sig + t;
   clk_mark(kp, sh, 0);
   beacon(kp, 2, t, 0);
   const int nP = load_parents(kp, P, sm, sh, o_begin, sh.o_end - o_begin, false);
+  trace_ev(kp, t, 1);
   const int E = sh.E;
   const bool oversize = E > kp.T;
   const uint32_t key0 = (uint32_t)o_begin + 1;
@@ -168,11 +174,10 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   }
   clk_mark(kp, sh, 2);
   beacon(kp, 4, t, 0);
-  trace_ev(kp, t, 1);
-  if (threadIdx.x == 0) {                       // own discovery done: LOCAL
-    __threadfence();                            // the block's atomicMin marks first
-    st_release_u64(&mine->word, LB_LOCAL);
-  }
+  trace_ev(kp, t, 2);
+  // own discovery done: LOCAL.  The release store orders the block's atomicMin
+  // marks (performed before discover's closing barrier) ahead of the flag.
+  if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL);
   // early Discovered: all predecessors already discovered?
   if (threadIdx.x < 32 && !oversize && !(kp.flags & F_NO_EARLY)) {
     int ready = 0;
@@ -184,7 +189,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   if (sh.aborted) return;
   const bool early = sh.s_early == 1;
   if (early) {
-    trace_ev(kp, t, 2);
+    trace_ev(kp, t, 3);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     rediscover(kp, P, sm, sh, o_begin, E);      // dense array after sorting
     count_outputs(kp, sm, sh, nP, E);
@@ -193,6 +198,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
       st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));   // early Counted
       stat_add(kp, &kp.stats->redisc_early, 1);
     }
+    trace_ev(kp, t, 4);
     clk_mark(kp, sh, 4);
     if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
     clk_mark(kp, sh, 5);
@@ -207,7 +213,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     __syncthreads();
     clk_mark(kp, sh, 3);
     if (sh.aborted) return;
-    trace_ev(kp, t, 2);
+    trace_ev(kp, t, 3);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     if (oversize) {
       oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
@@ -221,15 +227,15 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
       st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));
       stat_add(kp, &kp.stats->redisc_late, 1);
     }
+    trace_ev(kp, t, 4);
     clk_mark(kp, sh, 4);
   }
   // Counted: prefix over the predecessors' aggregates
   beacon(kp, 8, t, sh.count);
-  trace_ev(kp, t, 3);
+  trace_ev(kp, t, 5);
   if (threadIdx.x < 32) {
     int out_off = 0, q_off = 0;
     const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off);
-    if (threadIdx.x == 0) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[5] = 1000 + (int)ok; }
     if (threadIdx.x == 0) {
       if (!ok) {
         sh.aborted = 1;
@@ -249,7 +255,7 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
   if (sh.aborted) return;
   const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
   beacon(kp, 9, t, out_off);
-  trace_ev(kp, t, 4);
+  trace_ev(kp, t, 6);
   GenState g;
   if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; }
   if (oversize) {
@@ -258,11 +264,11 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
     if (kp.flags & F_NO_SORT) compact_segments(sm, sh, nP);
+    // write_output ends with a block barrier; thread 0's release stores of the
+    // new descriptors then publish the block's o[] writes cumulatively
     write_output(kp, P, sm, sh, nP, E, out_off);
-    __threadfence();
-    __syncthreads();
     clk_mark(kp, sh, 7);
-    trace_ev(kp, t, 5);
+    trace_ev(kp, t, 7);
     if (nb > 0) {
       build_prefix(kp, sm, sh, E);
       if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
@@ -277,11 +283,11 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
     stat_add(kp, &kp.stats->executed, 1);
   }
   __syncthreads();
-  trace_ev(kp, t, 6);
+  trace_ev(kp, t, 8);
 #ifdef RCM_TRACE
   if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
     for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
-      kp.trace[(size_t)(q_off + i) * 8 + 7] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
+      kp.trace[(size_t)(q_off + i) * kTraceW + kTraceW - 1] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
 #endif
   // empty slots: published as discovered with a zero aggregate
   const int emitted = sh.k;
@@ -298,22 +304,18 @@ __device__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm
       __threadfence();
       atomicExch(&kp.ctl->done, 1);
     } else {
-      // chain end: every reserved slot finished (each slot reserves before it
-      // counts itself; empties are counted by their generator)
-      __threadfence();
-      const int c = atomicAdd(&kp.ctl->completed, 1 + (nb - emitted)) + 1 + (nb - emitted);
-      if (c == ld_acquire_s32(&kp.ctl->qtail)) {
-        kp.ctl->incomplete = 1;
-        __threadfence();
-        atomicExch(&kp.ctl->done, 1);
-      }
+      // count this slot and the empties it generated as finished (each slot
+      // reserves before it counts itself).  Fire-and-forget: chain end without
+      // termination (completed == qtail) is detected by the idle dequeuers
+      // (lb_chain_exhausted), off this block's critical path.
+      red_release_add_s32(&kp.ctl->completed, 1 + (nb - emitted));
     }
   }
   __syncthreads();
   clk_mark(kp, sh, 8);
 }
 
-__device__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+__device__ __forceinline__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                              uint32_t epoch) {
   if (threadIdx.x == 0) {
     for (int i = 0; i < 10; ++i) sh.clk[i] = 0;

@@ -352,11 +352,27 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, un
 }
 
 // Dequeue the next non-empty batch in queue order.
+// Look-back chain end without termination (a disconnected graph): every
+// reserved slot has finished, so nothing will ever be published again.  A slot
+// counts itself (and the empties it generated) in `completed` only after its
+// reservation raised `qtail` (release), and every reserved slot is counted
+// exactly once, so completed == qtail read in this order (acquire) implies no
+// slot is still running.  Polled by blocks idling in dequeue.
+__device__ __noinline__ bool lb_chain_exhausted(const KParams& kp) {
+  const int c = ld_acquire_s32(&kp.ctl->completed);
+  if (c != ld_acquire_s32(&kp.ctl->qtail)) return false;
+  kp.ctl->incomplete = 1;   // idempotent: several idle blocks may get here
+  __threadfence();
+  atomicExch(&kp.ctl->done, 1);
+  return true;
+}
+
 // Thread 0; returns false when the chain is done.
 __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
   for (;;) {
     if (ld_relaxed_s32(&kp.ctl->done)) return false;
     const int t = atomicAdd(&kp.ctl->head, 1);
+    trace_ev(kp, t, 9);   // slot claimed (before its descriptor is seen)
     beacon(kp, 1, t, 0);
     if (t >= kp.qcap) {   // only possible after a capacity error; wait for done
       while (!ld_relaxed_s32(&kp.ctl->done)) __nanosleep(1000);
@@ -365,17 +381,19 @@ __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
     const Desc* d = kp.desc + t;
     uint64_t t0 = 0;
     unsigned ns = 0;
-    for (int it = 0; ld_acquire_u32(&d->tag) != epoch; ++it) {
+    for (int it = 0; ld_relaxed_u32(&d->tag) != epoch; ++it) {   // relaxed poll, acquire below
       if (ld_relaxed_s32(&kp.ctl->done)) return false;
       if (it >= 32) {
         __nanosleep(ns);
         if (ns < 512) ns = ns ? ns * 2 : 32;
       }
+      if ((it & 15) == 15 && !(kp.flags & F_SERIAL_CHAIN) && lb_chain_exhausted(kp)) return false;
       if ((it & 255) == 255) {
         if (t0 == 0) t0 = globaltimer();
         else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 1, t, ld_relaxed_s32(&kp.ctl->head), 0); return false; }
       }
     }
+    (void)ld_acquire_u32(&d->tag);   // acquire the publication (one L1 invalidation per dequeue)
     const int b = ld_relaxed_s32(&d->o_begin), e = ld_relaxed_s32(&d->o_end), nx = ld_relaxed_s32(&d->next);
     stat_add(kp, &kp.stats->dequeued, 1);
     if (b == e) { stat_add(kp, &kp.stats->empty, 1); continue; }
@@ -389,7 +407,7 @@ __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
 }
 
 // Process one dequeued batch of the chain: Alg. 5 BatchRCM.
-__device__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+__device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                             uint32_t epoch) {
   const int t = sh.t, o_begin = sh.o_begin, succ = sh.next;
   Sig* mine = kp.sig + t;
