@@ -330,6 +330,17 @@ extern "C" void rcm_plan_destroy(rcm_plan_t p) {
   delete p;
 }
 
+// k_main instantiation for `bps` resident blocks per SM (register budget
+// 64K / (bps * kThreads)); capped at 1024 threads per SM (64 registers).
+static const void* pick_kernel(int bps) {
+  constexpr int kMaxBps = 1024 / kThreads;   // >= 64 registers per thread
+  const int b = std::min(bps, kMaxBps);
+  if (b >= 4) return (const void*)k_main<(kMaxBps >= 4 ? 4 : 1)>;
+  if (b == 3) return (const void*)k_main<(kMaxBps >= 3 ? 3 : 1)>;
+  if (b == 2) return (const void*)k_main<(kMaxBps >= 2 ? 2 : 1)>;
+  return (const void*)k_main<1>;
+}
+
 extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t nnz_max,
                                         const rcm_options_t* opt_in) {
   if (!out || n_max <= 0 || nnz_max < 0 || n_max >= (1ll << 31) - 2) return RCM_ERR_INVALID_ARGUMENT;
@@ -338,7 +349,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   if (!p) return RCM_ERR_OUT_OF_MEMORY;
   if (opt_in) p->opt = *opt_in;
   rcm_options_t& o = p->opt;
-  if (o.batch_nodes < 0 || o.batch_nodes > kMaxBatchNodes || o.temp_elems < 0 || o.blocks_per_sm < 0 ||
+  if (o.batch_nodes < 0 || o.batch_nodes > kMaxBatchNodes || o.temp_elems < 0 || o.blocks_per_sm < 0 || o.blocks_per_sm > 4 ||
       o.validate < 0 || o.validate > 2 || o.queue_capacity < 0) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;
@@ -371,7 +382,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   p->T = T;
   p->smem = smem_bytes(p->BS, T);
   // one block per SM: the 128-register build (no spills); more: the 64-register build
-  p->kernel = bps == 1 ? (const void*)k_main<1> : (const void*)k_main<2>;
+  p->kernel = pick_kernel(bps);
   if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
     delete p;
     return RCM_ERR_CUDA;
@@ -380,7 +391,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, p->kernel, kThreads, p->smem);
   if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
   p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
-  if (p->nblocks > kThreads) p->nblocks = kThreads / p->num_sms * p->num_sms;   // block-0 scans assume <= kThreads
+  if (p->nblocks > kMaxBlocks) p->nblocks = kMaxBlocks / p->num_sms * p->num_sms;   // beacon / scratch sizing
   // queue bound: sum over generating batches of floor(N/B) + max(1, ceil(2V/T))
   const int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
   p->qcap = o.queue_capacity ? o.queue_capacity : std::min<int64_t>(qb, (1ll << 31) - 2);
@@ -411,7 +422,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   }
   AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
   AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
-  AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kThreads)); AL(p->w.sctl, 4 * 64);
+  AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kMaxBlocks)); AL(p->w.sctl, 4 * 64);
   AL(p->w.order, 4 * n); AL(p->w.lev, 4 * n); AL(p->w.front0, 4 * n); AL(p->w.front1, 4 * n);
   AL(p->w.gctl, 4 * 64); AL(p->w.gkey, 8 * 64);
 #undef AL

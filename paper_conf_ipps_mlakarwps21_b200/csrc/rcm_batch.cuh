@@ -82,13 +82,11 @@ struct SmemPtrs {
   int32_t* p_rs;              // BS row start (local, add ci_base)
   int32_t* p_eo;              // BS+1 edge-slot offsets (exclusive prefix of row lengths)
   int32_t* p_cnt;             // BS slots used (claims) per parent
-  int32_t* p_keep;            // BS kept children per parent
-  int32_t* p_out;             // BS+1 output offsets
 };
 
 __host__ __device__ inline size_t smem_bytes(int BS, int T) {
   return sizeof(unsigned long long) * (size_t)(T + 1) + sizeof(uint16_t) * (size_t)T + 16 +
-         sizeof(int32_t) * (size_t)(6 * BS + 2) + 64;
+         sizeof(int32_t) * (size_t)(4 * BS + 2) + 64;
 }
 
 __device__ inline SmemPtrs carve_smem(unsigned char* base, int BS, int T) {
@@ -104,14 +102,13 @@ __device__ inline SmemPtrs carve_smem(unsigned char* base, int BS, int T) {
   s.p_rs = ip + BS;
   s.p_eo = ip + 2 * BS;          // BS + 1
   s.p_cnt = ip + 3 * BS + 1;
-  s.p_keep = ip + 4 * BS + 1;
-  s.p_out = ip + 5 * BS + 1;     // BS + 1
   return s;
 }
 
 // Static shared state of one worker.
 struct ShState {
   unsigned long long wtmp64[kWarps + 1];
+  long long wtmp64b[kWarps + 1];
   int32_t wtmp32[kWarps + 1];
   long long wtmpll[kWarps + 1];
   int32_t t, o_begin, o_end, next;
@@ -244,18 +241,40 @@ __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm
   int lp = 0;
   unsigned long long* word = kp.word + P.node_base;
   const int32_t* col = kp.col_idx + P.ci_base;
-  for (int e = threadIdx.x; e < E; e += kThreads) {
-    lp = find_parent(sm.p_eo, lp, nP, e);
-    sm.lpof[e] = (uint16_t)lp;
-    int c = __ldg(col + sm.p_rs[lp] + (e - sm.p_eo[lp]));
-    uint32_t key = kfirst + (uint32_t)lp;
-    unsigned long long w = ld_relaxed_u64(word + c);
-    if ((uint32_t)(w >> 32) > key) {
-      unsigned long long old = atomicMin(word + c, ((unsigned long long)key << 32) | (w & 0xffffffffull));
-      uint32_t ow = (uint32_t)(old >> 32);
-      if (ow > key) {
-        int slot = sm.p_eo[lp] + atomicAdd(&sm.p_cnt[lp], 1);
-        sm.cand[slot] = ((old & 0xffffffffull) << 32) | (uint32_t)c;
+  // kDiscU edges per thread per round, each memory step issued for all of them
+  // before any result is used: the three dependent round trips (column,
+  // owner word, atomicMin) are paid once per round instead of once per edge.
+  for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
+    int c[kDiscU], lps[kDiscU];
+    unsigned long long w[kDiscU];
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) {
+      const int e = e0 + u * kThreads;
+      c[u] = -1;
+      if (e < E) {
+        lp = find_parent(sm.p_eo, lp, nP, e);
+        sm.lpof[e] = (uint16_t)lp;
+        lps[u] = lp;
+        c[u] = __ldg(col + sm.p_rs[lp] + (e - sm.p_eo[lp]));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) w[u] = c[u] >= 0 ? ld_weak_u64(word + c[u]) : 0ull;   // prefilter
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) {
+      const uint32_t key = kfirst + (uint32_t)lps[u];
+      if (c[u] >= 0 && (uint32_t)(w[u] >> 32) > key)
+        w[u] = atomicMin(word + c[u], ((unsigned long long)key << 32) | (w[u] & 0xffffffffull));
+      else
+        c[u] = -1;
+    }
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) {
+      const uint32_t key = kfirst + (uint32_t)lps[u];
+      const uint32_t ow = (uint32_t)(w[u] >> 32);
+      if (c[u] >= 0 && ow > key) {
+        int slot = sm.p_eo[lps[u]] + atomicAdd(&sm.p_cnt[lps[u]], 1);
+        sm.cand[slot] = ((w[u] & 0xffffffffull) << 32) | (uint32_t)c[u];
         steal |= (ow <= klast);   // taken from a sibling parent of this batch
         ++claims;
       }
@@ -266,35 +285,61 @@ __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm
     int tot = block_reduce_sum<int32_t>(claims, sh.wtmp32);
     if (threadIdx.x == 0 && tot) atomicAdd(&kp.stats->cand_spec, (unsigned long long)tot);
   }
-  for (int i = threadIdx.x; i < nP; i += kThreads) sm.p_keep[i] = sm.p_cnt[i];
   __syncthreads();
 }
 
 // ------------------------------------------------------------ rediscovery
-// Alg. 4 rediscover: drop n from c if a predecessor (or a sibling
-// parent with a smaller key) owns it now: keep iff owner(n) == key(p).
-// Removed candidates become kKeyMax (sorted to the end of their segment).
-__device__ int rediscover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
-                          int o_begin, int E) {
+// Alg. 4 rediscover fused with the count of the batch's outputs:
+// if `check`, drop n from c when a predecessor (or a sibling parent with a
+// smaller key) owns it now -- keep iff owner(n) == key(p); removed candidates
+// become kKeyMax.  Then sh.count = kept children and sh.V = the sum of their
+// valences clamped to Tg (oversize valences are clamped, they get
+// their own batch).  One combined block reduction.
+__device__ void rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                                 int o_begin, int E, bool check) {
   const unsigned long long* word = kp.word + P.node_base;
-  int removed = 0;
-  for (int e = threadIdx.x; e < E; e += kThreads) {
-    int lp = sm.lpof[e];
-    if (e - sm.p_eo[lp] >= sm.p_cnt[lp]) continue;
-    unsigned long long k = sm.cand[e];
-    if (k == kKeyMax) continue;
-    uint32_t c = (uint32_t)k;
-    uint32_t key = (uint32_t)o_begin + 1 + (uint32_t)lp;
-    if ((uint32_t)(ld_relaxed_u64(word + c) >> 32) != key) {
-      sm.cand[e] = kKeyMax;
-      atomicSub(&sm.p_keep[lp], 1);
-      ++removed;
+  long long kr = 0, val = 0;   // kept << 32 | removed, clamped valence sum
+  // kDiscU owner re-reads per thread in flight (see discover)
+  for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
+    unsigned long long k[kDiscU];
+    int lps[kDiscU];
+    uint32_t ow[kDiscU];
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) {
+      const int e = e0 + u * kThreads;
+      k[u] = kKeyMax;
+      if (e < E) {
+        const int lp = sm.lpof[e];
+        lps[u] = lp;
+        if (e - sm.p_eo[lp] < sm.p_cnt[lp]) k[u] = sm.cand[e];
+      }
+    }
+    if (check) {
+#pragma unroll
+      for (int u = 0; u < kDiscU; ++u)
+        ow[u] = k[u] != kKeyMax ? (uint32_t)(ld_weak_u64(word + (uint32_t)k[u]) >> 32) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < kDiscU; ++u) {
+      if (k[u] == kKeyMax) continue;
+      if (check && ow[u] != (uint32_t)o_begin + 1 + (uint32_t)lps[u]) {
+        sm.cand[e0 + u * kThreads] = kKeyMax;
+        kr += 1;
+      } else {
+        const long long d = (long long)(k[u] >> 32);
+        kr += 1ll << 32;
+        val += d < kp.Tg ? d : kp.Tg;
+      }
     }
   }
-  int tot = block_reduce_sum<int32_t>(removed, sh.wtmp32);
-  if (kp.collect_stats && threadIdx.x == 0 && tot)
-    atomicAdd(&kp.stats->cand_removed, (unsigned long long)tot);
-  return tot;
+  block_reduce_sum2(kr, val, sh.wtmpll, sh.wtmp64b);
+  if (threadIdx.x == 0) {
+    sh.count = (int)(kr >> 32);
+    sh.V = val;
+    sh.removed = (int)(kr & 0xffffffffll);
+    if (kp.collect_stats && sh.removed) atomicAdd(&kp.stats->cand_removed, (unsigned long long)sh.removed);
+  }
+  __syncthreads();
 }
 
 // ------------------------------------------------------------------ sort
@@ -395,64 +440,50 @@ __device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh
   __syncthreads();
 }
 
-// count = sum of kept children, V = sum of their valences clamped to T
-// (oversize valences are clamped, they get their own batch).
-// Kept children are the prefix [0, p_keep) of each (sorted) segment, or -- when
-// unsorted -- the non-kKeyMax entries of [0, p_cnt).
-__device__ void count_outputs(const KParams& kp, const SmemPtrs& sm, ShState& sh, int nP, int E) {
-  long long v = 0;
-  for (int e = threadIdx.x; e < E; e += kThreads) {
-    int lp = sm.lpof[e];
-    if (e - sm.p_eo[lp] >= sm.p_cnt[lp]) continue;
-    unsigned long long k = sm.cand[e];
-    if (k == kKeyMax) continue;
-    long long d = (long long)(k >> 32);
-    v += d < kp.Tg ? d : kp.Tg;
-  }
-  long long V = block_reduce_sum<long long>(v, sh.wtmpll);
-  int c = 0;
-  for (int lp = threadIdx.x; lp < nP; lp += kThreads) c += sm.p_keep[lp];
-  int C = block_reduce_sum<int32_t>(c, sh.wtmp32);
-  if (threadIdx.x == 0) { sh.count = C; sh.V = V; }
-  __syncthreads();
-}
-
-// Output (Alg. 5 ln 24-27): children in segment order at
-// o[out_off ...]; the RCM permutation is written reversed in the same pass
-// (perm[N-1-pos] = o[pos]) and optionally its inverse.
-// Requires sorted segments (kept = prefix of each segment).
+// Output (Alg. 5 ln 24-27): the kept children in array order
+// (parent segments in parent order, each sorted) at o[out_off ...]; the RCM
+// permutation is written reversed in the same pass (perm[N-1-pos] = o[pos],
+// P:L219) and optionally its inverse.  Kept = inside the parent's claims and
+// not removed (kKeyMax), so removed children need no re-sort.  One block scan
+// of (kept << 40 | clamped valence) over contiguous per-thread chunks gives
+// the positions; with `gen` the scan is also left in cand[0..E] for batch
+// generation (gen_chunk): cand[i] = exclusive prefix of slot i, cand[E] = total.
 __device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
-                             int nP, int E, int out_off) {
-  for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm.p_out[lp] = sm.p_keep[lp];
-  __syncthreads();
-  block_scan_array<int32_t>(sm.p_out, nP, sh.wtmp32);
+                             int E, int out_off, bool gen) {
+  const int per = (E + kThreads - 1) / kThreads;
+  const int b = threadIdx.x * per, e = min(E, b + per);
+  const unsigned long long Tg = (unsigned long long)kp.Tg;
+  unsigned long long s = 0;
+  for (int i = b; i < e; ++i) {
+    const int lp = sm.lpof[i];
+    const unsigned long long k = sm.cand[i];
+    if (i - sm.p_eo[lp] < sm.p_cnt[lp] && k != kKeyMax) {
+      const unsigned long long d = k >> 32;
+      s += (1ull << 40) | (d < Tg ? d : Tg);
+    }
+  }
+  unsigned long long tot;
+  unsigned long long run = block_exclusive_scan<unsigned long long>(s, sh.wtmp64, tot);
   int32_t* o = kp.o + P.o_base;
   int32_t* perm = kp.perm + P.perm_base;
   const int last = P.mat_n - 1;
-  for (int e = threadIdx.x; e < E; e += kThreads) {
-    int lp = sm.lpof[e];
-    int j = e - sm.p_eo[lp];
-    if (j >= sm.p_keep[lp]) continue;
-    int pos = out_off + sm.p_out[lp] + j;
-    int v = (int)(uint32_t)sm.cand[e];
-    o[pos] = v;
-    perm[last - pos] = v;
-    if (kp.iperm) kp.iperm[P.node_base + v] = last - pos;
+  for (int i = b; i < e; ++i) {
+    const int lp = sm.lpof[i];
+    const unsigned long long k = sm.cand[i];
+    unsigned long long x = 0;
+    if (i - sm.p_eo[lp] < sm.p_cnt[lp] && k != kKeyMax) {
+      const unsigned long long d = k >> 32;
+      x = (1ull << 40) | (d < Tg ? d : Tg);
+      const int pos = out_off + (int)(run >> 40);
+      const int v = (int)(uint32_t)k;
+      o[pos] = v;
+      perm[last - pos] = v;
+      if (kp.iperm) kp.iperm[P.node_base + v] = last - pos;
+    }
+    if (gen) sm.cand[i] = run;
+    run += x;
   }
-  __syncthreads();
-}
-
-// Unsorted variant (F_NO_SORT): kept = non-kKeyMax entries of each segment;
-// compact by a flat scan (order within a parent = discovery order).
-__device__ void compact_segments(const SmemPtrs& sm, ShState& sh, int nP) {
-  // per segment, move kept keys to the front (one thread per segment; debug path)
-  for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
-    unsigned long long* a = sm.cand + sm.p_eo[lp];
-    int w = 0;
-    for (int i = 0; i < sm.p_cnt[lp]; ++i)
-      if (a[i] != kKeyMax) a[w++] = a[i];
-    for (int i = w; i < sm.p_cnt[lp]; ++i) a[i] = kKeyMax;
-  }
+  if (gen && threadIdx.x == 0) sm.cand[E] = tot;
   __syncthreads();
 }
 
@@ -542,36 +573,6 @@ __device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, i
     ++g.emitted;
     g.has_pend = 0;
   }
-}
-
-// Build pre[] over this batch's slots in cand[] (after write_output), in place.
-__device__ void build_prefix(const KParams& kp, const SmemPtrs& sm, ShState& sh, int E) {
-  // each thread: contiguous chunk of slots; kept = j < p_keep[lp] (sorted segments)
-  const int per = (E + kThreads - 1) / kThreads;
-  const int b = threadIdx.x * per, e = min(E, b + per);
-  unsigned long long s = 0;
-  for (int i = b; i < e; ++i) {
-    int lp = sm.lpof[i];
-    if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
-      unsigned long long d = sm.cand[i] >> 32;
-      s += (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
-    }
-  }
-  unsigned long long tot;
-  unsigned long long run = block_exclusive_scan<unsigned long long>(s, sh.wtmp64, tot);
-  for (int i = b; i < e; ++i) {
-    int lp = sm.lpof[i];
-    unsigned long long x = 0;
-    if (i - sm.p_eo[lp] < sm.p_keep[lp]) {
-      unsigned long long d = sm.cand[i] >> 32;
-      x = (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
-    }
-    sm.cand[i] = run;
-    run += x;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) sm.cand[E] = tot;
-  __syncthreads();
 }
 
 // Publish empty batches q_off + [from, nb) (all threads of warp 0).

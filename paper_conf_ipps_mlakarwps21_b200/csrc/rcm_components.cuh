@@ -286,10 +286,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   }
   grid_barrier(kp);
   if (blockIdx.x == 0) {
-    const int x = threadIdx.x < kp.nblocks ? __ldcg(w.hist + threadIdx.x) : 0;
-    int tot;
-    const int ex = block_exclusive_scan<int32_t>(x, sh.wtmp32, tot);
-    if (threadIdx.x < kp.nblocks) w.hist[kp.nblocks + threadIdx.x] = ex;
+    const int tot = block_scan_partials<int32_t>(w.hist, w.hist + kp.nblocks, kp.nblocks, sh.wtmp32);
     if (threadIdx.x == 0) { w.sctl[0] = tot; w.sctl[1] = 0; }
   }
   grid_barrier(kp);
@@ -331,10 +328,8 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   }
   grid_barrier(kp);
   if (blockIdx.x == 0) {
-    const long long x = threadIdx.x < kp.nblocks ? __ldcg(w.offs + threadIdx.x) : 0;
-    long long tot;
-    const long long ex = block_exclusive_scan<long long>(x, sh.wtmpll, tot);
-    if (threadIdx.x < kp.nblocks) w.hist[threadIdx.x] = (int)ex;   // block bases (counts < 2^31)
+    // block bases (counts < 2^31)
+    block_scan_partials<long long, int32_t>(w.offs, w.hist, kp.nblocks, sh.wtmpll);
     if (threadIdx.x == 0) {
       kp.ctl->n_comp = count;
       kp.ctl->n_chain = 0;

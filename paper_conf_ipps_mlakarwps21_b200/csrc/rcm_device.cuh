@@ -13,9 +13,10 @@ constexpr int kThreads = RCM_THREADS;       // threads per persistent worker blo
 constexpr int kWarps = kThreads / 32;
 static_assert(kThreads % 32 == 0 && kThreads >= 256 && kThreads <= 1024, "block size");
 #ifndef RCM_DISC_U
-#define RCM_DISC_U 8
+#define RCM_DISC_U 4
 #endif
 constexpr int kDiscU = RCM_DISC_U;          // edge slots per thread in flight in discovery
+constexpr int kMaxBlocks = 1024;            // persistent workers per launch (beacon / scratch sizing)
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner
 constexpr uint64_t kKeyMax = ~0ull;         // removed / padding sort key
@@ -160,6 +161,12 @@ __device__ __forceinline__ void st_release_s32(int32_t* p, int32_t v) {
 __device__ __forceinline__ void st_relaxed_s32(int32_t* p, int32_t v) {
   asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// Owner-word load the compiler may schedule freely (a plain ld.global.cg, L2,
+// not volatile): for prefilters and rediscovery re-reads, where a batch of
+// independent loads is issued before any result is used.  Owner keys only
+// decrease (atomicMin), so a stale value is never below the current one; it
+// stays ordered by barriers and fences like any other load.
+__device__ __forceinline__ unsigned long long ld_weak_u64(const unsigned long long* p) { return __ldcg(p); }
 // L2-coherent load for data written by other blocks during this launch.
 __device__ __forceinline__ int32_t ld_cg_s32(const int32_t* p) { return __ldcg(p); }
 
@@ -209,6 +216,40 @@ __device__ __forceinline__ T block_reduce_sum(T v, T* warp_tmp) {
   T tot;
   block_exclusive_scan<T>(v, warp_tmp, tot);
   return tot;
+}
+
+// Block-wide sums of two values with one pair of barriers (all threads get both).
+__device__ __forceinline__ void block_reduce_sum2(long long& a, long long& b, long long* ta, long long* tb) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) {
+    a += __shfl_xor_sync(0xffffffffu, a, d);
+    b += __shfl_xor_sync(0xffffffffu, b, d);
+  }
+  if (lane == 0) { ta[wid] = a; tb[wid] = b; }
+  __syncthreads();
+  a = 0;
+  b = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; ++w) { a += ta[w]; b += tb[w]; }   // broadcast reads
+  __syncthreads();
+}
+
+// Exclusive scan of m per-block partials in global memory (in[] and out[]
+// distinct), by one block in chunks of kThreads (m may exceed the block size).
+// Returns the total.
+template <typename T, typename U = T>
+__device__ __forceinline__ T block_scan_partials(const T* in, U* out, int m, T* warp_tmp) {
+  T carry = 0;
+  for (int base = 0; base < m; base += kThreads) {
+    const int i = base + threadIdx.x;
+    const T x = i < m ? __ldcg(in + i) : T(0);
+    T tot;
+    const T ex = block_exclusive_scan<T>(x, warp_tmp, tot);
+    if (i < m) out[i] = (U)(carry + ex);
+    carry += tot;
+  }
+  return carry;
 }
 
 // Exclusive scan, in place, of a[0..len) in shared memory; returns the total.

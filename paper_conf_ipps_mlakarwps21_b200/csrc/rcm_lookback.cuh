@@ -191,8 +191,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   if (early) {
     trace_ev(kp, t, 3);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
-    rediscover(kp, P, sm, sh, o_begin, E);      // dense array after sorting
-    count_outputs(kp, sm, sh, nP, E);
+    rediscover_count(kp, P, sm, sh, o_begin, E, true);   // before sorting: removed sort to the end
     if (threadIdx.x == 0) {
       sh.nb = lb_nb(kp, sh.count, sh.V);
       st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));   // early Counted
@@ -218,9 +217,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     if (oversize) {
       oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
     } else {
-      const int removed = rediscover(kp, P, sm, sh, o_begin, E);
-      if (removed && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
-      count_outputs(kp, sm, sh, nP, E);
+      rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
     }
     if (threadIdx.x == 0) {
       sh.nb = lb_nb(kp, sh.count, sh.V);
@@ -263,16 +260,12 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
-    if (kp.flags & F_NO_SORT) compact_segments(sm, sh, nP);
     // write_output ends with a block barrier; thread 0's release stores of the
     // new descriptors then publish the block's o[] writes cumulatively
-    write_output(kp, P, sm, sh, nP, E, out_off);
+    write_output(kp, P, sm, sh, E, out_off, nb > 0);
     clk_mark(kp, sh, 7);
     trace_ev(kp, t, 7);
-    if (nb > 0) {
-      build_prefix(kp, sm, sh, E);
-      if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
-    }
+    if (nb > 0 && threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
   }
   if (threadIdx.x == 0) {
     if (nb > 0) {

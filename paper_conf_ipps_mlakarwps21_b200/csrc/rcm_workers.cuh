@@ -439,12 +439,9 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
       __threadfence();   // the block's atomicMin marks before the signal
       send_sig(succ_sig, S_DISCOVERED);
     }
-    if (s_early < S_DISCOVERED || sh.steal) {
-      rediscover(kp, P, sm, sh, o_begin, E);
-      if (threadIdx.x == 0 && s_early < S_DISCOVERED) stat_add(kp, &kp.stats->redisc_early, 1);
-    }
+    rediscover_count(kp, P, sm, sh, o_begin, E, s_early < S_DISCOVERED || sh.steal);
+    if (threadIdx.x == 0 && s_early < S_DISCOVERED) stat_add(kp, &kp.stats->redisc_early, 1);
     rediscovered = true;
-    count_outputs(kp, sm, sh, nP, E);
     if (threadIdx.x == 0) {
       const unsigned long long w = load_sig(mine);
       if (sig_state(w) >= S_COUNTED) signal_count(kp, sh, mine, w, succ_sig, succ);
@@ -465,9 +462,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     if (oversize) {
       oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
     } else {
-      const int removed = rediscover(kp, P, sm, sh, o_begin, E);
-      if (removed && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // move removed to the end
-      count_outputs(kp, sm, sh, nP, E);
+      rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
     }
     if (threadIdx.x == 0) {
       stat_add(kp, &kp.stats->redisc_late, 1);
@@ -509,8 +504,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     oversize_output(kp, P, sm, sh, out_off, gen, g, sh.q_off, sh.nb, epoch);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
-    if (kp.flags & F_NO_SORT) compact_segments(sm, sh, nP);
-    write_output(kp, P, sm, sh, nP, E, out_off);
+    write_output(kp, P, sm, sh, E, out_off, gen);
     __threadfence();
     __syncthreads();
     if (threadIdx.x == 0 && need_completed && sig_state(sh.sigw) < S_COMPLETED) {
@@ -518,10 +512,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     }
     __syncthreads();
     if (sh.aborted) return;
-    if (gen) {
-      build_prefix(kp, sm, sh, E);
-      if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, sh.q_off, sh.nb, epoch);
-    }
+    if (gen && threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, sh.q_off, sh.nb, epoch);
   }
   if (threadIdx.x == 0) {
     if (sh.fwd) send_sig(succ_sig, sig_pack(out_off + sh.count, sh.q_off, 1, S_COMPLETED));
@@ -695,13 +686,10 @@ __device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm
     } else {
       if (threadIdx.x == 0) sh.steal = 0;
       discover(kp, P, sm, sh, pos, nP, E);
-      if (sh.steal) rediscover(kp, P, sm, sh, pos, E);
+      rediscover_count(kp, P, sm, sh, pos, E, sh.steal != 0);
+      const int c = sh.count;
       if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
-      else compact_segments(sm, sh, nP);
-      int c = 0;
-      for (int lp = threadIdx.x; lp < nP; lp += kThreads) c += sm.p_keep[lp];
-      c = block_reduce_sum<int32_t>(c, sh.wtmp32);
-      write_output(kp, P, sm, sh, nP, E, written);
+      write_output(kp, P, sm, sh, E, written, false);
       written += c;
     }
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->executed, 1);
