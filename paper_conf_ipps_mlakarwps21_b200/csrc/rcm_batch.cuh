@@ -501,6 +501,7 @@ struct GenState {
   int emitted;     // batches written so far
   int pend_b, pend_e;  // last closed batch, not yet written (its `next` is unknown)
   int has_pend;
+  int defer;       // 1: write descriptor fields only; the caller fences and writes the tags
 };
 
 __device__ __forceinline__ void publish_desc(Desc* d, int b, int e, int next, uint32_t epoch) {
@@ -510,11 +511,16 @@ __device__ __forceinline__ void publish_desc(Desc* d, int b, int e, int next, ui
   st_release_u32(&d->tag, epoch);   // release: orders the fields above (and, cumulatively, what the block wrote before its last barrier)
 }
 
+__device__ __forceinline__ void write_desc(const GenState& g, Desc* d, int b, int e, int next, uint32_t epoch) {
+  if (g.defer) { d->o_begin = b; d->o_end = e; d->next = next; }
+  else publish_desc(d, b, e, next, epoch);
+}
+
 __device__ __forceinline__ void gen_close(const KParams& kp, GenState& g, int end, int q_off,
                                           int nb, uint32_t epoch) {
   if (g.has_pend) {
     if (g.emitted < nb)   // never exceeded; guarded anyway
-      publish_desc(kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + g.emitted + 1, epoch);
+      write_desc(g, kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + g.emitted + 1, epoch);
     else
       latch_error(kp.ctl, ST_CAPACITY);
     ++g.emitted;
@@ -568,7 +574,7 @@ __device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, i
                            uint32_t epoch) {
   if (g.cnt > 0) gen_close(kp, g, end, q_off, nb, epoch);
   if (g.has_pend) {
-    if (g.emitted < nb) publish_desc(kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + nb, epoch);
+    if (g.emitted < nb) write_desc(g, kp.desc + q_off + g.emitted, g.pend_b, g.pend_e, q_off + nb, epoch);
     else latch_error(kp.ctl, ST_CAPACITY);
     ++g.emitted;
     g.has_pend = 0;

@@ -21,15 +21,19 @@
 
 namespace rcm {
 
-constexpr unsigned long long LB_LOCAL = 1, LB_DINCL = 2, LB_AGG = 4;
-
-// a-word: flags | count << 3 (31 bit) | nb << 34 (30 bit)
-__device__ __forceinline__ unsigned long long lb_a(int count, int nb, unsigned long long flags) {
-  return flags | ((unsigned long long)(uint32_t)count << 3) | ((unsigned long long)(uint32_t)nb << 34);
+// Sig::word: Discovered flags, release stores (they order the block's
+// atomicMin marks, cumulatively, before the flag).
+constexpr unsigned long long LB_LOCAL = 1, LB_DINCL = 2;
+// Sig::ovh holds the Counted facts, plain values (relaxed stores, no fence):
+//   AGG  = 2 | count << 2 (31 bit) | nb << 33 (30 bit)
+//   INCL = 1 | out_end << 2 (31 bit) | q_end << 33 (30 bit), replaces AGG
+// A successor reads one word per slot; nothing it reads depends on other data.
+constexpr unsigned long long LB_INCL = 1, LB_AGG = 2;
+__device__ __forceinline__ unsigned long long lb_pfx(unsigned long long kind, long long a, long long b) {
+  return kind | ((unsigned long long)(uint32_t)a << 2) | ((unsigned long long)(uint32_t)b << 33);
 }
-// b-word: INCL | out_end << 1 (31 bit) | q_end << 32
-__device__ __forceinline__ unsigned long long lb_b(int out_end, int q_end) {
-  return 1ull | ((unsigned long long)(uint32_t)out_end << 1) | ((unsigned long long)(uint32_t)q_end << 32);
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ void lb_spin(unsigned& ns, int it) {
@@ -99,17 +103,16 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
     const bool valid = idx >= 0;
     // relaxed: the prefix needs only the values carried in the status words
     const unsigned long long b = valid ? ld_relaxed_u64(&kp.sig[idx].ovh) : 0ull;
-    const unsigned long long a = valid ? ld_relaxed_u64(&kp.sig[idx].word) : 0ull;
-    const unsigned incl = __ballot_sync(0xffffffffu, !valid || (b & 1ull));
-    const unsigned agg = __ballot_sync(0xffffffffu, valid && (a & LB_AGG));
+    const unsigned incl = __ballot_sync(0xffffffffu, !valid || (b & LB_INCL));
+    const unsigned agg = __ballot_sync(0xffffffffu, valid && (b & LB_AGG));
     const int stop = incl ? __ffs(incl) - 1 : 32;
     const unsigned need = stop == 32 ? 0xffffffffu : ((1u << stop) - 1);
     unsigned take = need;
     const bool complete = (agg & need) == need;
     if (!complete) take = (1u << (__ffs(~agg & need) - 1)) - 1;   // AGG prefix of the window
     // accumulate the AGG lanes in `take`
-    long long c = ((take >> lane) & 1) ? (long long)((a >> 3) & 0x7fffffffull) : 0;
-    long long q = ((take >> lane) & 1) ? (long long)(a >> 34) : 0;
+    long long c = ((take >> lane) & 1) ? (long long)((b >> 2) & 0x7fffffffull) : 0;
+    long long q = ((take >> lane) & 1) ? (long long)(b >> 33) : 0;
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) {
       c += __shfl_xor_sync(0xffffffffu, c, d);
@@ -121,7 +124,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
       if (stop < 32) {
         const unsigned long long bs = __shfl_sync(0xffffffffu, b, stop);
         const int vs = __shfl_sync(0xffffffffu, (int)valid, stop);
-        if (vs) { base_out = (long long)((bs >> 1) & 0x7fffffffull); base_q = (long long)(bs >> 32); }
+        if (vs) { base_out = (long long)((bs >> 2) & 0x7fffffffull); base_q = (long long)(bs >> 33); }
         j = -1;
         break;
       }
@@ -135,7 +138,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
     int quit = lane == 0 && (ld_relaxed_s32(&kp.ctl->status) || (count == 0 && ld_relaxed_s32(&kp.ctl->done)));
     if ((it & 1023) == 1023 && lane == 0) {
       if (t0 == 0) t0 = globaltimer();
-      else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 3, t, j, (long long)a); quit = 1; }
+      else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 3, t, j, (long long)b); quit = 1; }
     }
     if (__shfl_sync(0xffffffffu, quit, 0)) return false;   // warp-uniform exit
     lb_spin(ns, it);
@@ -194,7 +197,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     rediscover_count(kp, P, sm, sh, o_begin, E, true);   // before sorting: removed sort to the end
     if (threadIdx.x == 0) {
       sh.nb = lb_nb(kp, sh.count, sh.V);
-      st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));   // early Counted
+      st_relaxed_u64(&mine->ovh, lb_pfx(LB_AGG, sh.count, sh.nb));   // early Counted
       stat_add(kp, &kp.stats->redisc_early, 1);
     }
     trace_ev(kp, t, 4);
@@ -221,7 +224,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     }
     if (threadIdx.x == 0) {
       sh.nb = lb_nb(kp, sh.count, sh.V);
-      st_release_u64(&mine->word, lb_a(sh.count, sh.nb, LB_LOCAL | LB_DINCL | LB_AGG));
+      st_relaxed_u64(&mine->ovh, lb_pfx(LB_AGG, sh.count, sh.nb));
       stat_add(kp, &kp.stats->redisc_late, 1);
     }
     trace_ev(kp, t, 4);
@@ -240,7 +243,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
         sh.out_off = out_off;
         sh.q_off = q_off;
         if ((long long)q_off + sh.nb > kp.qcap) { latch_error(kp.ctl, ST_CAPACITY); sh.nb = 0; sh.aborted = 1; }
-        st_release_u64(&mine->ovh, lb_b(out_off + sh.count, q_off + sh.nb));
+        st_relaxed_u64(&mine->ovh, lb_pfx(LB_INCL, out_off + sh.count, q_off + sh.nb));
         atomicMax(&kp.ctl->qtail, q_off + sh.nb);
         atomicMax(&kp.ctl->chain_total, out_off + sh.count);
         stat_add(kp, &kp.stats->generated, sh.nb);
@@ -254,56 +257,55 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   beacon(kp, 9, t, out_off);
   trace_ev(kp, t, 6);
   GenState g;
-  if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; }
+  if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; g.defer = !oversize; }
   if (oversize) {
     if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) return;
     oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
-    // write_output ends with a block barrier; thread 0's release stores of the
-    // new descriptors then publish the block's o[] writes cumulatively
+    // write_output ends with a block barrier: the block's o[] writes precede
+    // thread 0's fence below, which publishes them cumulatively
     write_output(kp, P, sm, sh, E, out_off, nb > 0);
     clk_mark(kp, sh, 7);
     trace_ev(kp, t, 7);
     if (nb > 0 && threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
   }
   if (threadIdx.x == 0) {
+    int emitted = 0;
     if (nb > 0) {
-      gen_finish(kp, g, out_off + sh.count, q_off, nb, epoch);
+      gen_finish(kp, g, out_off + sh.count, q_off, nb, epoch);   // descriptor fields only (deferred tags)
       if (g.emitted > nb) latch_error(kp.ctl, ST_CAPACITY);
+      emitted = min(g.emitted, nb);
     }
-    sh.k = nb > 0 ? g.emitted : 0;
+    // empty slots: discovered, zero aggregate (values only)
+    for (int i = emitted; i < nb; ++i) {
+      st_relaxed_u64(&kp.sig[q_off + i].word, LB_LOCAL);
+      st_relaxed_u64(&kp.sig[q_off + i].ovh, lb_pfx(LB_AGG, 0, 0));
+      Desc* d = kp.desc + q_off + i;
+      d->o_begin = 0; d->o_end = 0; d->next = q_off + i + 1;
+    }
     stat_add(kp, &kp.stats->executed, 1);
-  }
-  __syncthreads();
-  trace_ev(kp, t, 8);
-#ifdef RCM_TRACE
-  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
-    for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
-      kp.trace[(size_t)(q_off + i) * kTraceW + kTraceW - 1] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
-#endif
-  // empty slots: published as discovered with a zero aggregate
-  const int emitted = sh.k;
-  if (nb > emitted && threadIdx.x < 32) {
-    for (int i = emitted + threadIdx.x; i < nb; i += 32) {
-      st_release_u64(&kp.sig[q_off + i].word, LB_LOCAL | LB_AGG);
-      publish_desc(kp.desc + q_off + i, 0, 0, q_off + i + 1, epoch);
-    }
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
     const int total = out_off + sh.count;
+    // one fence publishes the o[] writes and every descriptor's fields; the
+    // tags (and the completion count) are then relaxed stores (release pattern)
+    fence_acquire_gpu();
+    for (int i = 0; i < nb; ++i) st_relaxed_u32(&kp.desc[q_off + i].tag, epoch);
     if (total == P.pos0 + P.size) {             // early termination
-      __threadfence();
       atomicExch(&kp.ctl->done, 1);
     } else {
       // count this slot and the empties it generated as finished (each slot
       // reserves before it counts itself).  Fire-and-forget: chain end without
       // termination (completed == qtail) is detected by the idle dequeuers
       // (lb_chain_exhausted), off this block's critical path.
-      red_release_add_s32(&kp.ctl->completed, 1 + (nb - emitted));
+      red_relaxed_add_s32(&kp.ctl->completed, 1 + (nb - emitted));
     }
   }
+  trace_ev(kp, t, 8);
+#ifdef RCM_TRACE
+  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
+    for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
+      kp.trace[(size_t)(q_off + i) * kTraceW + kTraceW - 1] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;
+#endif
   __syncthreads();
   clk_mark(kp, sh, 8);
 }

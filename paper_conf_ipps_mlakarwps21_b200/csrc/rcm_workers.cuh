@@ -489,6 +489,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     g.val = sh.ovh_t;
     g.emitted = 0;
     g.has_pend = 0;
+    g.defer = 0;
   }
   const bool gen = !sh.fwd && sh.nb > 0;
   // wait(Completed) before publishing batches that reference an overhang, or
