@@ -173,8 +173,7 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
 template <int kMinBlocks>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_constant__ KParams kp, const __grid_constant__ MainArgs a) {
   __shared__ ShState sh;
-  extern __shared__ __align__(16) unsigned char dsm[];
-  SmemPtrs sm = carve_smem(dsm, kp.BS, kp.T);
+  SmemPtrs sm;   // layout accessors sm_*(kp) (rcm_batch.cuh)
   const int G = gthreads(kp);
   // ---- phase 0: reset the per-call control state
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -217,7 +216,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
     }
     if (gtid() == 0) { a.w.sctl[0] = a.num_mats; a.w.sctl[1] = 0; }
     grid_barrier(kp);
-    radix_sort_phase(kp, a.w, 0, 64, reinterpret_cast<int32_t*>(sm.cand), sh);
+    radix_sort_phase(kp, a.w, 0, 64, reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
     const int32_t* order = ld_cg_s32(a.w.sctl + 1) ? a.w.vals1 : a.w.vals0;
     Problem* solos = const_cast<Problem*>(kp.solos);
     for (int i = gtid(); i < a.num_mats; i += G) {
@@ -361,20 +360,20 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
-  p->BS = o.batch_nodes ? o.batch_nodes : 256;
+  const bool dense = !o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max;
+  // dense rows (FEM-like): smaller batches shorten the critical generation
+  // chain
+  p->BS = o.batch_nodes ? o.batch_nodes : dense ? 160 : 256;
   const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
   const size_t static_sh = sizeof(ShState) + 64;
-  // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per block)
+  // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per
+  // block), 10 B per slot (candidate key, local parent id)
   const size_t per_block =
       std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
   int T = o.temp_elems;
   if (!T) T = (int)((per_block - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
-  if (!o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max) {
-    // dense rows (FEM-like): smaller batches shorten the critical generation
-    // chain, and the shared memory left over serves as L1
-    T = std::min(T, 6144);
-    p->BS = 160;
-  }
+  // dense: B_s rows of ~27 fit; the shared memory left over serves as L1
+  if (dense) T = std::min(T, 6144);
   if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;

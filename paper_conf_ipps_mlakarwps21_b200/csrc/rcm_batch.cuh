@@ -74,35 +74,35 @@ __device__ __forceinline__ void beacon(const KParams& kp, int phase, int slot, i
 enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16,
                  F_LEVELED = 32 };
 
-// Dynamic shared memory of one worker.
-struct SmemPtrs {
-  unsigned long long* cand;   // T+1 candidate keys (valence << 32 | id); reused for prefixes
-  uint16_t* lpof;             // T local parent id of every edge slot
-  int32_t* p_v;               // BS parent ids
-  int32_t* p_rs;              // BS row start (local, add ci_base)
-  int32_t* p_eo;              // BS+1 edge-slot offsets (exclusive prefix of row lengths)
-  int32_t* p_cnt;             // BS slots used (claims) per parent
-};
+
+// Dynamic shared memory of one worker.  The layout is recomputed from the
+// kernel parameters (constant bank) at every use instead of being held in
+// registers:
+//   cand  T+1 candidate keys (valence << 32 | id); reused for prefixes
+//   lpof  T local parent id of every edge slot (u16)
+//   p_v   BS parent ids
+//   p_rs  BS row starts (local, add ci_base)
+//   p_eo  BS+1 edge-slot offsets (exclusive prefix of row lengths)
+//   p_cnt BS slots used (claims) per parent
+extern __shared__ __align__(16) unsigned char rcm_dsm[];
+struct SmemPtrs {};
+__device__ __forceinline__ unsigned long long* sm_cand(const KParams&) {
+  return reinterpret_cast<unsigned long long*>(rcm_dsm);
+}
+__device__ __forceinline__ uint16_t* sm_lpof(const KParams& kp) {
+  return reinterpret_cast<uint16_t*>(rcm_dsm + 8 * ((size_t)kp.T + 1));
+}
+__device__ __forceinline__ int32_t* sm_ip(const KParams& kp) {
+  return reinterpret_cast<int32_t*>(rcm_dsm + ((8 * ((size_t)kp.T + 1) + 2 * (size_t)kp.T + 15) & ~size_t(15)));
+}
+__device__ __forceinline__ int32_t* sm_p_v(const KParams& kp) { return sm_ip(kp); }
+__device__ __forceinline__ int32_t* sm_p_rs(const KParams& kp) { return sm_ip(kp) + kp.BS; }
+__device__ __forceinline__ int32_t* sm_p_eo(const KParams& kp) { return sm_ip(kp) + 2 * kp.BS; }        // BS + 1
+__device__ __forceinline__ int32_t* sm_p_cnt(const KParams& kp) { return sm_ip(kp) + 3 * kp.BS + 1; }
 
 __host__ __device__ inline size_t smem_bytes(int BS, int T) {
-  return sizeof(unsigned long long) * (size_t)(T + 1) + sizeof(uint16_t) * (size_t)T + 16 +
+  return sizeof(unsigned long long) * (size_t)(T + 1) + 2 * (size_t)T + 16 +
          sizeof(int32_t) * (size_t)(4 * BS + 2) + 64;
-}
-
-__device__ inline SmemPtrs carve_smem(unsigned char* base, int BS, int T) {
-  SmemPtrs s;
-  size_t off = 0;
-  s.cand = reinterpret_cast<unsigned long long*>(base);
-  off += sizeof(unsigned long long) * (size_t)(T + 1);
-  s.lpof = reinterpret_cast<uint16_t*>(base + off);
-  off += sizeof(uint16_t) * (size_t)T;
-  off = (off + 15) & ~size_t(15);
-  int32_t* ip = reinterpret_cast<int32_t*>(base + off);
-  s.p_v = ip;
-  s.p_rs = ip + BS;
-  s.p_eo = ip + 2 * BS;          // BS + 1
-  s.p_cnt = ip + 3 * BS + 1;
-  return s;
 }
 
 // Static shared state of one worker.
@@ -189,13 +189,13 @@ __device__ int load_parents(const KParams& kp, const Problem& P, const SmemPtrs&
     int v = ld_cg_s32(kp.o + P.o_base + o_begin + lp);
     const int32_t* rp = kp.row_ptr + P.rp_base + v;
     int rs = __ldg(rp), re = __ldg(rp + 1);
-    sm.p_v[lp] = v;
-    sm.p_rs[lp] = rs;
-    sm.p_eo[lp] = re - rs;
+    sm_p_v(kp)[lp] = v;
+    sm_p_rs(kp)[lp] = rs;
+    sm_p_eo(kp)[lp] = re - rs;
   }
   __syncthreads();
-  int E = block_scan_array<int32_t>(sm.p_eo, nP, sh.wtmp32);
-  sm.p_eo[nP] = E;   // (visible after the barrier below)
+  int E = block_scan_array<int32_t>(sm_p_eo(kp), nP, sh.wtmp32);
+  sm_p_eo(kp)[nP] = E;   // (visible after the barrier below)
   __syncthreads();
   if (cut_T && E > kp.T && nP > 1) {
     // largest nP' with p_eo[nP'] <= T (p_eo is non-decreasing); at least 1.
@@ -203,15 +203,24 @@ __device__ int load_parents(const KParams& kp, const Problem& P, const SmemPtrs&
       int lo = 1, hi = nP;   // p_eo[lo] may exceed T when the first row alone is oversize
       while (lo < hi) {
         int mid = (lo + hi + 1) >> 1;
-        if (sm.p_eo[mid] <= kp.T) lo = mid; else hi = mid - 1;
+        if (sm_p_eo(kp)[mid] <= kp.T) lo = mid; else hi = mid - 1;
       }
       sh.nP = lo;
     }
     __syncthreads();
     nP = sh.nP;
-    E = sm.p_eo[nP];
+    E = sm_p_eo(kp)[nP];
   }
   if (threadIdx.x == 0) { sh.nP = nP; sh.E = E; }
+  // local parent of every edge slot, one warp per parent (discovery and the
+  // later passes read it instead of searching p_eo per slot)
+  if (E <= kp.T) {
+    const int lane = threadIdx.x & 31;
+    for (int lp = threadIdx.x >> 5; lp < nP; lp += kWarps) {
+      const int eb = sm_p_eo(kp)[lp], ee = sm_p_eo(kp)[lp + 1];
+      for (int j = eb + lane; j < ee; j += 32) sm_lpof(kp)[j] = (uint16_t)lp;
+    }
+  }
   __syncthreads();
   return nP;
 }
@@ -234,11 +243,10 @@ __device__ __forceinline__ int find_parent(const int32_t* p_eo, int lo, int nP, 
 // of the scratchpad ("atomicAdd to reserve a unique spot").
 __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                          int o_begin, int nP, int E) {
-  for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm.p_cnt[lp] = 0;
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm_p_cnt(kp)[lp] = 0;
   __syncthreads();
   const uint32_t kfirst = (uint32_t)o_begin + 1, klast = (uint32_t)o_begin + (uint32_t)nP;
   int steal = 0, claims = 0;
-  int lp = 0;
   unsigned long long* word = kp.word + P.node_base;
   const int32_t* col = kp.col_idx + P.ci_base;
   // kDiscU edges per thread per round, each memory step issued for all of them
@@ -252,10 +260,9 @@ __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm
       const int e = e0 + u * kThreads;
       c[u] = -1;
       if (e < E) {
-        lp = find_parent(sm.p_eo, lp, nP, e);
-        sm.lpof[e] = (uint16_t)lp;
+        const int lp = sm_lpof(kp)[e];
         lps[u] = lp;
-        c[u] = __ldg(col + sm.p_rs[lp] + (e - sm.p_eo[lp]));
+        c[u] = __ldg(col + sm_p_rs(kp)[lp] + (e - sm_p_eo(kp)[lp]));
       }
     }
 #pragma unroll
@@ -273,8 +280,8 @@ __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm
       const uint32_t key = kfirst + (uint32_t)lps[u];
       const uint32_t ow = (uint32_t)(w[u] >> 32);
       if (c[u] >= 0 && ow > key) {
-        int slot = sm.p_eo[lps[u]] + atomicAdd(&sm.p_cnt[lps[u]], 1);
-        sm.cand[slot] = ((w[u] & 0xffffffffull) << 32) | (uint32_t)c[u];
+        int slot = sm_p_eo(kp)[lps[u]] + atomicAdd(&sm_p_cnt(kp)[lps[u]], 1);
+        sm_cand(kp)[slot] = ((w[u] & 0xffffffffull) << 32) | (uint32_t)c[u];
         steal |= (ow <= klast);   // taken from a sibling parent of this batch
         ++claims;
       }
@@ -299,34 +306,35 @@ __device__ void rediscover_count(const KParams& kp, const Problem& P, const Smem
                                  int o_begin, int E, bool check) {
   const unsigned long long* word = kp.word + P.node_base;
   long long kr = 0, val = 0;   // kept << 32 | removed, clamped valence sum
-  // kDiscU owner re-reads per thread in flight (see discover)
+  // kDiscU owner re-reads per thread in flight (see discover); only the owner
+  // keys stay in registers, the slots are re-read from shared memory
   for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
-    unsigned long long k[kDiscU];
-    int lps[kDiscU];
     uint32_t ow[kDiscU];
+    if (check) {
+#pragma unroll
+      for (int u = 0; u < kDiscU; ++u) {
+        const int e = e0 + u * kThreads;
+        ow[u] = 0;
+        if (e < E) {
+          const int lp = sm_lpof(kp)[e];
+          const unsigned long long k = sm_cand(kp)[e];
+          if (e - sm_p_eo(kp)[lp] < sm_p_cnt(kp)[lp] && k != kKeyMax)
+            ow[u] = (uint32_t)(ld_weak_u64(word + (uint32_t)k) >> 32);
+        }
+      }
+    }
 #pragma unroll
     for (int u = 0; u < kDiscU; ++u) {
       const int e = e0 + u * kThreads;
-      k[u] = kKeyMax;
-      if (e < E) {
-        const int lp = sm.lpof[e];
-        lps[u] = lp;
-        if (e - sm.p_eo[lp] < sm.p_cnt[lp]) k[u] = sm.cand[e];
-      }
-    }
-    if (check) {
-#pragma unroll
-      for (int u = 0; u < kDiscU; ++u)
-        ow[u] = k[u] != kKeyMax ? (uint32_t)(ld_weak_u64(word + (uint32_t)k[u]) >> 32) : 0u;
-    }
-#pragma unroll
-    for (int u = 0; u < kDiscU; ++u) {
-      if (k[u] == kKeyMax) continue;
-      if (check && ow[u] != (uint32_t)o_begin + 1 + (uint32_t)lps[u]) {
-        sm.cand[e0 + u * kThreads] = kKeyMax;
+      if (e >= E) continue;
+      const int lp = sm_lpof(kp)[e];
+      const unsigned long long k = sm_cand(kp)[e];
+      if (e - sm_p_eo(kp)[lp] >= sm_p_cnt(kp)[lp] || k == kKeyMax) continue;
+      if (check && ow[u] != (uint32_t)o_begin + 1 + (uint32_t)lp) {
+        sm_cand(kp)[e] = kKeyMax;
         kr += 1;
       } else {
-        const long long d = (long long)(k[u] >> 32);
+        const long long d = (long long)(k >> 32);
         kr += 1ll << 32;
         val += d < kp.Tg ? d : kp.Tg;
       }
@@ -389,9 +397,9 @@ __device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh
   if (threadIdx.x == 0) sh.big_n = 0;
   __syncthreads();
   for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
-    int n = sm.p_cnt[lp];
+    int n = sm_p_cnt(kp)[lp];
     if (n <= 1) continue;
-    unsigned long long* a = sm.cand + sm.p_eo[lp];
+    unsigned long long* a = sm_cand(kp) + sm_p_eo(kp)[lp];
     if (n <= 16) {
       for (int i = 1; i < n; ++i) {
         unsigned long long x = a[i];
@@ -412,29 +420,29 @@ __device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh
     // warp-level for segments <= 4096, the rest block-level below
     for (int b = wid; b < nbig; b += kWarps) {
       int lp = sh.big_list[b];
-      int n = sm.p_cnt[lp];
+      int n = sm_p_cnt(kp)[lp];
       if (n > 4096) continue;
-      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, lane, 32, [] { __syncwarp(); });
+      bitonic_sort_flip(sm_cand(kp) + sm_p_eo(kp)[lp], n, lane, 32, [] { __syncwarp(); });
     }
     __syncthreads();
     for (int b = 0; b < nbig; ++b) {
       int lp = sh.big_list[b];
-      int n = sm.p_cnt[lp];
+      int n = sm_p_cnt(kp)[lp];
       if (n <= 4096) continue;
-      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
+      bitonic_sort_flip(sm_cand(kp) + sm_p_eo(kp)[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
     }
   } else {
     // too many large segments for the list: one warp per segment, scanning all
     for (int lp = wid; lp < nP; lp += kWarps) {
-      int n = sm.p_cnt[lp];
+      int n = sm_p_cnt(kp)[lp];
       if (n <= 16 || n > 4096) continue;
-      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, lane, 32, [] { __syncwarp(); });
+      bitonic_sort_flip(sm_cand(kp) + sm_p_eo(kp)[lp], n, lane, 32, [] { __syncwarp(); });
     }
     __syncthreads();
     for (int lp = 0; lp < nP; ++lp) {
-      int n = sm.p_cnt[lp];
+      int n = sm_p_cnt(kp)[lp];
       if (n <= 4096) continue;
-      bitonic_sort_flip(sm.cand + sm.p_eo[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
+      bitonic_sort_flip(sm_cand(kp) + sm_p_eo(kp)[lp], n, threadIdx.x, kThreads, [] { __syncthreads(); });
     }
   }
   __syncthreads();
@@ -455,9 +463,9 @@ __device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs
   const unsigned long long Tg = (unsigned long long)kp.Tg;
   unsigned long long s = 0;
   for (int i = b; i < e; ++i) {
-    const int lp = sm.lpof[i];
-    const unsigned long long k = sm.cand[i];
-    if (i - sm.p_eo[lp] < sm.p_cnt[lp] && k != kKeyMax) {
+    const int lp = sm_lpof(kp)[i];
+    const unsigned long long k = sm_cand(kp)[i];
+    if (i - sm_p_eo(kp)[lp] < sm_p_cnt(kp)[lp] && k != kKeyMax) {
       const unsigned long long d = k >> 32;
       s += (1ull << 40) | (d < Tg ? d : Tg);
     }
@@ -468,10 +476,10 @@ __device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs
   int32_t* perm = kp.perm + P.perm_base;
   const int last = P.mat_n - 1;
   for (int i = b; i < e; ++i) {
-    const int lp = sm.lpof[i];
-    const unsigned long long k = sm.cand[i];
+    const int lp = sm_lpof(kp)[i];
+    const unsigned long long k = sm_cand(kp)[i];
     unsigned long long x = 0;
-    if (i - sm.p_eo[lp] < sm.p_cnt[lp] && k != kKeyMax) {
+    if (i - sm_p_eo(kp)[lp] < sm_p_cnt(kp)[lp] && k != kKeyMax) {
       const unsigned long long d = k >> 32;
       x = (1ull << 40) | (d < Tg ? d : Tg);
       const int pos = out_off + (int)(run >> 40);
@@ -480,10 +488,10 @@ __device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs
       perm[last - pos] = v;
       if (kp.iperm) kp.iperm[P.node_base + v] = last - pos;
     }
-    if (gen) sm.cand[i] = run;
+    if (gen) sm_cand(kp)[i] = run;
     run += x;
   }
-  if (gen && threadIdx.x == 0) sm.cand[E] = tot;
+  if (gen && threadIdx.x == 0) sm_cand(kp)[E] = tot;
   __syncthreads();
 }
 

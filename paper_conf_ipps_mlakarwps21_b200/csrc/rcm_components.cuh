@@ -314,7 +314,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   int maxdeg = ld_cg_s32(&kp.ctl->maxdeg);
   int dbits = 0;
   while (dbits < 32 && (1ll << dbits) <= maxdeg) ++dbits;
-  radix_sort_phase(kp, w, a.idbits, a.idbits + dbits, reinterpret_cast<int32_t*>(sm.cand), sh);
+  radix_sort_phase(kp, w, a.idbits, a.idbits + dbits, reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
   // offsets: exclusive scan of sizes in key order, after the chain-first total
   const int count = ld_cg_s32(w.sctl);
   const int cur = ld_cg_s32(w.sctl + 1);

@@ -15,7 +15,8 @@ static_assert(kThreads % 32 == 0 && kThreads >= 256 && kThreads <= 1024, "block 
 #ifndef RCM_DISC_U
 #define RCM_DISC_U 4
 #endif
-constexpr int kDiscU = RCM_DISC_U;          // edge slots per thread in flight in discovery
+constexpr int kDiscU = RCM_DISC_U;
+          // edge slots per thread in flight in discovery
 constexpr int kMaxBlocks = 1024;            // persistent workers per launch (beacon / scratch sizing)
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner

@@ -85,7 +85,7 @@ __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const Proble
     }
     if (gtid() == 0) w.sctl[1] = 0;
     grid_barrier(kp);
-    radix_sort_phase(kp, w, 0, tot, reinterpret_cast<int32_t*>(sm.cand), sh);   // parallelSort (ln 14)
+    radix_sort_phase(kp, w, 0, tot, reinterpret_cast<int32_t*>(sm_cand(kp)), sh);   // parallelSort (ln 14)
     const unsigned long long* keys = ld_cg_s32(w.sctl + 1) ? w.keys1 : w.keys0;
     const unsigned long long idmask = (1ull << idbits) - 1;
     for (int i = gtid(); i < cnt; i += G) {                                     // parallelWrite (ln 15)

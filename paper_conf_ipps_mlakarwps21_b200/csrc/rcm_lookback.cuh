@@ -171,7 +171,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   __syncthreads();
   clk_mark(kp, sh, 1);
   if (oversize) {
-    if (!oversize_discover(kp, P, sm, sh, key0, sm.p_rs[0], E)) return;
+    if (!oversize_discover(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E)) return;
   } else {
     discover(kp, P, sm, sh, o_begin, nP, E);
   }
@@ -218,7 +218,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     trace_ev(kp, t, 3);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     if (oversize) {
-      oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
+      oversize_rediscover_count(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E);
     } else {
       rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
     }
@@ -259,7 +259,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   GenState g;
   if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; g.defer = !oversize; }
   if (oversize) {
-    if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) return;
+    if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) return;
     oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
@@ -268,7 +268,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     write_output(kp, P, sm, sh, E, out_off, nb > 0);
     clk_mark(kp, sh, 7);
     trace_ev(kp, t, 7);
-    if (nb > 0 && threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, q_off, nb, epoch);
+    if (nb > 0 && threadIdx.x == 0) gen_chunk(kp, g, sm_cand(kp), E, out_off, q_off, nb, epoch);
   }
   if (threadIdx.x == 0) {
     int emitted = 0;
@@ -302,6 +302,10 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   }
   trace_ev(kp, t, 8);
 #ifdef RCM_TRACE
+  if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && t < kp.trace_cap) {
+    kp.trace[(size_t)t * kTraceW + 10] = (unsigned long long)(uint32_t)ld_relaxed_s32(&kp.ctl->head);
+    kp.trace[(size_t)t * kTraceW + 11] = (unsigned long long)(uint32_t)q_off;
+  }
   if (kp.collect_stats == 3 && threadIdx.x == 0 && kp.trace && nb > 0)
     for (int i = 0; i < nb && q_off + i < kp.trace_cap; ++i)
       kp.trace[(size_t)(q_off + i) * kTraceW + kTraceW - 1] = ((unsigned long long)(uint32_t)t << 32) | blockIdx.x;

@@ -154,7 +154,7 @@ __device__ void block_radix_sort_global(unsigned long long* a, unsigned long lon
 // (valence, id) there, written out, and cut into batches chunk by chunk.
 __device__ bool oversize_discover(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                   ShState& sh, uint32_t key, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm.cand);
+  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
   if (nw > 2 * (kp.T + 1)) {
     if (threadIdx.x == 0) latch_error(kp.ctl, ST_CAPACITY);
@@ -185,7 +185,7 @@ __device__ bool oversize_discover(const KParams& kp, const Problem& P, const Sme
 // Rediscover (keep iff owner == key), then count and clamped valence sum.
 __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                           ShState& sh, uint32_t key, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm.cand);
+  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
   const unsigned long long* word = kp.word + P.node_base;
   const int32_t* col = kp.col_idx + P.ci_base + rs;
@@ -217,7 +217,7 @@ __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, c
 // Gather kept children into spill, sort them.  Returns false on capacity error.
 __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                      ShState& sh, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm.cand);
+  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
   const int C = sh.count;
   if (threadIdx.x == 0) {
@@ -251,7 +251,7 @@ __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const 
   __syncthreads();
   // sort by (valence, id); the bitmap area is free now
   block_radix_sort_global(out, kp.spill + kp.spill_cap + sh.spill_base, C,
-                          reinterpret_cast<int32_t*>(sm.cand), sh);
+                          reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
   return true;
 }
 
@@ -288,12 +288,12 @@ __device__ void oversize_output(const KParams& kp, const Problem& P, const SmemP
     unsigned long long run = block_exclusive_scan<unsigned long long>(s, sh.wtmp64, tot);
     for (int i = b; i < e; ++i) {
       unsigned long long d = __ldcg(src + c0 + i) >> 32;
-      sm.cand[i] = run;
+      sm_cand(kp)[i] = run;
       run += (1ull << 40) | (d < (unsigned long long)kp.Tg ? d : (unsigned long long)kp.Tg);
     }
-    if (threadIdx.x == 0) sm.cand[m] = tot;
+    if (threadIdx.x == 0) sm_cand(kp)[m] = tot;
     __syncthreads();
-    if (threadIdx.x == 0) gen_chunk(kp, g, sm.cand, m, out_off + c0, q_off, nb, epoch);
+    if (threadIdx.x == 0) gen_chunk(kp, g, sm_cand(kp), m, out_off + c0, q_off, nb, epoch);
     __syncthreads();
   }
 }
@@ -424,7 +424,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
   const bool oversize = E > kp.T;   // only single-node batches (batch generation)
   const uint32_t key0 = (uint32_t)o_begin + 1;
   if (oversize) {
-    if (!oversize_discover(kp, P, sm, sh, key0, sm.p_rs[0], E)) return;
+    if (!oversize_discover(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E)) return;
   } else {
     discover(kp, P, sm, sh, o_begin, nP, E);                                    // ln 3
   }
@@ -460,7 +460,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     __syncthreads();
     if (sh.aborted) return;
     if (oversize) {
-      oversize_rediscover_count(kp, P, sm, sh, key0, sm.p_rs[0], E);
+      oversize_rediscover_count(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E);
     } else {
       rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
     }
@@ -496,7 +496,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
   // before forwarding Completed for an overhang we passed on (ln 27-29)
   const bool need_completed = sh.fwd || sh.ovh_n > 0;
   if (oversize) {
-    if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) return;
+    if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) return;
     if (threadIdx.x == 0 && need_completed && sig_state(sh.sigw) < S_COMPLETED) {
       if (sig_state(wait_sig(mine, S_COMPLETED, kp.ctl)) < S_COMPLETED) sh.aborted = 1;
     }
@@ -513,7 +513,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
     }
     __syncthreads();
     if (sh.aborted) return;
-    if (gen && threadIdx.x == 0) gen_chunk(kp, g, sm.cand, E, out_off, sh.q_off, sh.nb, epoch);
+    if (gen && threadIdx.x == 0) gen_chunk(kp, g, sm_cand(kp), E, out_off, sh.q_off, sh.nb, epoch);
   }
   if (threadIdx.x == 0) {
     if (sh.fwd) send_sig(succ_sig, sig_pack(out_off + sh.count, sh.q_off, 1, S_COMPLETED));
@@ -677,9 +677,9 @@ __device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm
     const int E = sh.E;
     if (E > kp.T) {
       const uint32_t key = (uint32_t)pos + 1;
-      if (!oversize_discover(kp, P, sm, sh, key, sm.p_rs[0], E)) break;
-      oversize_rediscover_count(kp, P, sm, sh, key, sm.p_rs[0], E);
-      if (!oversize_gather_sort(kp, P, sm, sh, sm.p_rs[0], E)) break;
+      if (!oversize_discover(kp, P, sm, sh, key, sm_p_rs(kp)[0], E)) break;
+      oversize_rediscover_count(kp, P, sm, sh, key, sm_p_rs(kp)[0], E);
+      if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) break;
       GenState g;
       oversize_output(kp, P, sm, sh, written, false, g, 0, 0, 0);
       if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);

@@ -24,6 +24,8 @@ cnt = min(st["batches_generated"] + 2, 1 << 20)
 buf = (ctypes.c_ulonglong * (W * cnt))()
 lib.rcm_debug_trace(plan.handle, cnt, buf)
 tr = np.frombuffer(buf, dtype=np.uint64).reshape(cnt, W).astype(np.int64)
+if len(sys.argv) > 3:
+    np.save(sys.argv[3], tr)   # raw trace for offline analysis
 real = np.nonzero(tr[:, 0])[0]
 t0 = tr[real, 0].min()
 ev = (tr[real, :10] - t0) / 1000.0          # us
@@ -53,6 +55,8 @@ print("along chain mean us:", {n: round(float(np.mean(dd[:, i])), 2) for i, n in
       "of which no free block", round(float(np.mean(claim_late)), 2) if pick else None)
 # batch sizes along the chain vs overall
 sizes = None
+hq = [int(tr[s, 10]) - int(tr[s, 11]) for s in chain]
+print("head - q_off at chain publishes: median", int(np.median(hq)), "min", min(hq), "max", max(hq))
 print("chain total us", round(ev[rows[-1], 8] - ev[rows[0], 0], 1))
 # in-flight slots (claimed, not finished) sampled at every chain publish
 fin = ev[:, 8]; clm = ev[:, 9]

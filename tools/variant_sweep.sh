@@ -1,6 +1,7 @@
 #!/bin/bash
 mkdir -p gpurun_out
-RCM_LIB=build/librcm_trace.so timeout 300 python tools/trace_timeline.py 2 '{}' 25 > gpurun_out/timeline_c2.txt 2>&1
-timeout 600 python tools/sweep.py 2 '[{}, {"batch_nodes": 96, "temp_elems": 6144}, {"batch_nodes": 128, "temp_elems": 6144}, {"batch_nodes": 256, "temp_elems": 6144}, {"batch_nodes": 256, "temp_elems": 8192}, {"batch_nodes": 160, "temp_elems": 4608}]' 7 > gpurun_out/sw4_c2.jsonl 2> gpurun_out/sw4_c2.err
-timeout 600 python tools/sweep.py 3 '[{}, {"batch_nodes": 128}, {"batch_nodes": 512}, {"batch_nodes": 256, "temp_elems": 6144}]' 7 > gpurun_out/sw4_c3.jsonl 2> gpurun_out/sw4_c3.err
-timeout 600 python tools/sweep.py 4 '[{}, {"batch_nodes": 128}, {"batch_nodes": 512}]' 7 > gpurun_out/sw4_c4.jsonl 2> gpurun_out/sw4_c4.err
+timeout 900 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1
+for c in 2 3 4; do
+  timeout 300 python tools/sweep.py $c '[{}]' 9 > gpurun_out/sw11_c$c.jsonl 2> gpurun_out/sw11_c$c.err
+done
+RCM_LIB=build/librcm_trace.so timeout 300 python tools/trace_chain.py 2 "{}" gpurun_out/trace11_c2.npy > gpurun_out/trace11_c2.txt 2>&1
