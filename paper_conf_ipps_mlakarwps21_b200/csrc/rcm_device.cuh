@@ -17,6 +17,13 @@ static_assert(kThreads % 32 == 0 && kThreads >= 256 && kThreads <= 1024, "block 
 #endif
 constexpr int kDiscU = RCM_DISC_U;
           // edge slots per thread in flight in discovery
+// spin back-off caps (ns): dequeue polling, look-back polling
+#ifndef RCM_DQ_SLEEP_MAX
+#define RCM_DQ_SLEEP_MAX 512
+#endif
+#ifndef RCM_LB_SLEEP_MAX
+#define RCM_LB_SLEEP_MAX 256
+#endif
 constexpr int kMaxBlocks = 1024;            // persistent workers per launch (beacon / scratch sizing)
 constexpr int kMaxBatchNodes = 1024;        // B_s upper bound (u16 local parent ids)
 constexpr uint32_t kInf = 0xFFFFFFFFu;      // "unmarked" owner

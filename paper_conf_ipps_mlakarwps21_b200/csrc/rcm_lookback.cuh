@@ -39,7 +39,7 @@ __device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned l
 __device__ __forceinline__ void lb_spin(unsigned& ns, int it) {
   if (it >= 16) {
     __nanosleep(ns);
-    if (ns < 256) ns = ns ? ns * 2 : 32;
+    if (ns < RCM_LB_SLEEP_MAX) ns = ns ? ns * 2 : 32;
   }
 }
 

@@ -385,7 +385,7 @@ __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
       if (ld_relaxed_s32(&kp.ctl->done)) return false;
       if (it >= 32) {
         __nanosleep(ns);
-        if (ns < 512) ns = ns ? ns * 2 : 32;
+        if (ns < RCM_DQ_SLEEP_MAX) ns = ns ? ns * 2 : 32;
       }
       if ((it & 15) == 15 && !(kp.flags & F_SERIAL_CHAIN) && lb_chain_exhausted(kp)) return false;
       if ((it & 255) == 255) {
