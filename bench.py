@@ -103,6 +103,11 @@ def load_workload(cfg: int):
     raise ValueError(cfg)
 
 
+def _plan_env() -> dict:
+    """Plan options from RCM_PLAN (JSON), for tuning sweeps; empty by default."""
+    return json.loads(os.environ["RCM_PLAN"]) if os.environ.get("RCM_PLAN") else {}
+
+
 def traffic_from_profile(cfg: int):
     p = os.path.join(ROOT, "profiles", f"traffic_c{cfg}.json")
     if os.path.exists(p):
@@ -191,7 +196,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     rp = rp_h.to(dev)
     ci = ci_h.to(dev)
     perm = torch.empty(n, dtype=torch.int32, device=dev)
-    plan = rcm.Plan(n, nnz, collect_stats=0)
+    plan = rcm.Plan(n, nnz, collect_stats=0, **_plan_env())
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
@@ -350,7 +355,7 @@ def run_ours_c5(args, rank: int, world: int, local_rank: int):
     mine = parts[rank]
     b = sd.c5_generate(mine, num=num, device=dev)
     total, total_nnz = b["total"], b["total_nnz"]
-    plan = rcm.Plan(total, total_nnz)
+    plan = rcm.Plan(total, total_nnz, **_plan_env())
     perm = torch.empty(total, dtype=torch.int32, device=dev)
     stream = torch.cuda.current_stream()
     part_tot = [int(n_all[p].sum()) for p in parts]
