@@ -183,6 +183,27 @@ def run_reference_c5(args):
 
 
 # ----------------------------------------------------------------- our arm
+def cpu_batch_context(g, mode, start, ref, runs: int = 3):
+    """The paper's CPU-BATCH (NEXT-4, libcpubatch.so: Alg. 5 on std::thread) on
+    every host core, full workload, median of `runs`: context for the paper's
+    multicore numbers, not a baseline of the GPU kernel."""
+    try:
+        from paper_conf_ipps_mlakarwps21_b200 import cpu_batch
+        cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
+        ts, ok = [], True
+        for _ in range(runs):
+            t0 = time.perf_counter()
+            perm = cpu_batch.rcm_cpu_batch(g.row_ptr, g.col_idx, mode, start, threads=cores)
+            ts.append(time.perf_counter() - t0)
+            ok = ok and bool(np.array_equal(perm, ref))
+        sec = statistics.median(ts)
+        return {"value": round(g.n / sec / 1e6, 3), "unit": "Mnodes/s", "cores": cores, "kind": "cpu_batch",
+                "ms": round(1e3 * sec, 3), "parity_vs_oracle": "bit-identical" if ok else "MISMATCH",
+                "sample": f"full workload graph, median of {runs} runs"}
+    except Exception as exc:   # context only: never fails the bench line
+        return {"unavailable": str(exc)[:200]}
+
+
 def run_ours(args, rank: int, world: int, local_rank: int):
     import torch
     import paper_conf_ipps_mlakarwps21_b200 as rcm
@@ -316,6 +337,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                          "kind": "oracle", "ms": round(o_ms, 3),
                          "sample": "full workload graph, serial oracle, median of 3 runs"},
         "speedup_vs_oracle": round(o_ms / ms, 2),
+        "cpu_batch": cpu_batch_context(g, mode, start, ref) if rank == 0 else None,
         "e2e": {"value": round(e2e_val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 4 * (n + 1) + 4 * nnz,
                 "d2h_bytes_per_step": 4 * n, "ms_per_step": round(e2e_ms / args.steps, 4)},
         "gpu_launches": args.steps,

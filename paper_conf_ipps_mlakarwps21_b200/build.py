@@ -44,5 +44,23 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+CPU_LIB = os.path.join(HERE, "libcpubatch.so")
+CPU_SRC = os.path.join(CSRC, "cpu_batch.cpp")
+CXX = os.environ.get("CXX", "g++")
+
+
+def build_cpu(force: bool = False) -> str:
+    """Host CPU-BATCH (NEXT-4, include/rcm_cpu.h): plain C++17 + std::thread."""
+    hdr = os.path.join(HERE, "..", "include", "rcm_cpu.h")
+    if (not force and os.path.exists(CPU_LIB)
+            and os.path.getmtime(CPU_LIB) >= max(os.path.getmtime(CPU_SRC), os.path.getmtime(hdr))):
+        return CPU_LIB
+    tmp = CPU_LIB + f".tmp{os.getpid()}"
+    subprocess.check_call([CXX, "-O3", "-std=c++17", "-shared", "-fPIC", "-pthread", "-o", tmp, CPU_SRC])
+    os.replace(tmp, CPU_LIB)
+    return CPU_LIB
+
+
 if __name__ == "__main__":
+    print(build_cpu(force="--force" in sys.argv))
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
