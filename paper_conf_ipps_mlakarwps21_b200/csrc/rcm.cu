@@ -126,7 +126,9 @@ __device__ void prologue_batched_phase(const KParams& kp, const MainArgs& a) {
 
 // The scheduling phase: every chain problem in turn on all blocks (grid
 // barrier between chains), then the solo problems, one per block at a time.
-__device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
+template <bool kMB>
+__device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh,
+                                               ShState& sh2) {
   const int nchain = ld_cg_s32(&kp.ctl->n_chain);
   for (int c = 0; c < nchain; ++c) {
     if (kp.chains[c].flags & 2) {   // PSEUDO_PERIPHERAL component: GL seed first (C-5)
@@ -146,7 +148,8 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
     // instead of pinning 16 registers across the whole traversal
     if (threadIdx.x == 0) sh.prob = kp.chains[c];
     __syncthreads();
-    chain_worker(kp, sh.prob, sm, sh, epoch);
+    if constexpr (kMB) chain_worker_mb(kp, sh.prob, sm, sh, sh2, epoch);
+    else chain_worker(kp, sh.prob, sm, sh, epoch);
     grid_barrier(kp);
     chain_reset_signals(kp);
     grid_barrier(kp);
@@ -170,10 +173,12 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
 
 // One launch per call: reset -> prologue -> seed / problem set-up ->
 // traversal -> (components -> traversal).  Grid barriers between phases.
-template <int kMinBlocks>
+template <int kMinBlocks, bool kMB>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_constant__ KParams kp, const __grid_constant__ MainArgs a) {
   __shared__ ShState sh;
+  __shared__ ShState sh2;   // second batch context (multi-batch execution, kMB only)
   SmemPtrs sm;   // layout accessors sm_*(kp) (rcm_batch.cuh)
+  if (threadIdx.x == 0) rcm_ctx_base = 0;
   const int G = gthreads(kp);
   // ---- phase 0: reset the per-call control state
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -250,13 +255,13 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
   grid_barrier(kp);
   stamp(kp, 2);
   // ---- phase 3: the traversal (a2-a12)
-  schedule_phase(kp, a, sm, sh);
+  schedule_phase<kMB>(kp, a, sm, sh, sh2);
   grid_barrier(kp);
   stamp(kp, 3);
   // ---- phase 4: components left over by the chain-first pass (a13)
   if (!a.batched && !a.solo && ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
     cc_phase(kp, a, sm, sh);
-    schedule_phase(kp, a, sm, sh);
+    schedule_phase<kMB>(kp, a, sm, sh, sh2);
     grid_barrier(kp);
   }
   stamp(kp, 4);
@@ -331,13 +336,14 @@ extern "C" void rcm_plan_destroy(rcm_plan_t p) {
 
 // k_main instantiation for `bps` resident blocks per SM (register budget
 // 64K / (bps * kThreads)); capped at 1024 threads per SM (64 registers).
-static const void* pick_kernel(int bps) {
+static const void* pick_kernel(int bps, bool mb) {
   constexpr int kMaxBps = 1024 / kThreads;   // >= 64 registers per thread
   const int b = std::min(bps, kMaxBps);
-  if (b >= 4) return (const void*)k_main<(kMaxBps >= 4 ? 4 : 1)>;
-  if (b == 3) return (const void*)k_main<(kMaxBps >= 3 ? 3 : 1)>;
-  if (b == 2) return (const void*)k_main<(kMaxBps >= 2 ? 2 : 1)>;
-  return (const void*)k_main<1>;
+  if (mb) return b >= 2 ? (const void*)k_main<(kMaxBps >= 2 ? 2 : 1), true> : (const void*)k_main<1, true>;
+  if (b >= 4) return (const void*)k_main<(kMaxBps >= 4 ? 4 : 1), false>;
+  if (b == 3) return (const void*)k_main<(kMaxBps >= 3 ? 3 : 1), false>;
+  if (b == 2) return (const void*)k_main<(kMaxBps >= 2 ? 2 : 1), false>;
+  return (const void*)k_main<1, false>;
 }
 
 extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t nnz_max,
@@ -365,13 +371,14 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   // chain
   p->BS = o.batch_nodes ? o.batch_nodes : dense ? 160 : 256;
   const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
-  const size_t static_sh = sizeof(ShState) + 64;
+  const size_t static_sh = 2 * sizeof(ShState) + 64;
+  const int nctx = (o.flags & RCM_FLAG_MULTI_BATCH) ? 2 : 1;   // batch contexts per block
   // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per
   // block), 10 B per slot (candidate key, local parent id)
   const size_t per_block =
       std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
   int T = o.temp_elems;
-  if (!T) T = (int)((per_block - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
+  if (!T) T = (int)((per_block / nctx - 16 - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
   // dense: B_s rows of ~27 fit; the shared memory left over serves as L1
   if (dense) T = std::min(T, 6144);
   if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
@@ -379,9 +386,9 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
     return RCM_ERR_INVALID_ARGUMENT;
   }
   p->T = T;
-  p->smem = smem_bytes(p->BS, T);
+  p->smem = nctx == 1 ? smem_bytes(p->BS, T) : nctx * ((smem_bytes(p->BS, T) + 15) & ~size_t(15));
   // one block per SM: the 128-register build (no spills); more: the 64-register build
-  p->kernel = pick_kernel(bps);
+  p->kernel = pick_kernel(bps, nctx == 2);
   if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
     delete p;
     return RCM_ERR_CUDA;

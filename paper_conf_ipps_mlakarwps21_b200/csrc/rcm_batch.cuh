@@ -72,7 +72,7 @@ __device__ __forceinline__ void beacon(const KParams& kp, int phase, int slot, i
 }
 
 enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN = 8, F_SERIAL_CHAIN = 16,
-                 F_LEVELED = 32 };
+                 F_LEVELED = 32, F_MULTI_BATCH = 64 };
 
 
 // Dynamic shared memory of one worker.  The layout is recomputed from the
@@ -85,15 +85,21 @@ enum : int32_t { F_NO_OVERHANG = 1, F_NO_EARLY = 2, F_NO_SORT = 4, F_FORCE_CHAIN
 //   p_eo  BS+1 edge-slot offsets (exclusive prefix of row lengths)
 //   p_cnt BS slots used (claims) per parent
 extern __shared__ __align__(16) unsigned char rcm_dsm[];
+// multi-batch execution (F_MULTI_BATCH): byte offset of the current batch
+// context's scratch (0 or the context size); always 0 otherwise
+__shared__ uint32_t rcm_ctx_base;
 struct SmemPtrs {};
-__device__ __forceinline__ unsigned long long* sm_cand(const KParams&) {
-  return reinterpret_cast<unsigned long long*>(rcm_dsm);
+__device__ __forceinline__ unsigned char* sm_base(const KParams& kp) {
+  return rcm_dsm + rcm_ctx_base;
+}
+__device__ __forceinline__ unsigned long long* sm_cand(const KParams& kp) {
+  return reinterpret_cast<unsigned long long*>(sm_base(kp));
 }
 __device__ __forceinline__ uint16_t* sm_lpof(const KParams& kp) {
-  return reinterpret_cast<uint16_t*>(rcm_dsm + 8 * ((size_t)kp.T + 1));
+  return reinterpret_cast<uint16_t*>(sm_base(kp) + 8 * ((size_t)kp.T + 1));
 }
 __device__ __forceinline__ int32_t* sm_ip(const KParams& kp) {
-  return reinterpret_cast<int32_t*>(rcm_dsm + ((8 * ((size_t)kp.T + 1) + 2 * (size_t)kp.T + 15) & ~size_t(15)));
+  return reinterpret_cast<int32_t*>(sm_base(kp) + ((8 * ((size_t)kp.T + 1) + 2 * (size_t)kp.T + 15) & ~size_t(15)));
 }
 __device__ __forceinline__ int32_t* sm_p_v(const KParams& kp) { return sm_ip(kp); }
 __device__ __forceinline__ int32_t* sm_p_rs(const KParams& kp) { return sm_ip(kp) + kp.BS; }
@@ -114,6 +120,7 @@ struct ShState {
   int32_t t, o_begin, o_end, next;
   int32_t nP, E, steal, removed;
   int32_t s_early, s_mid, counted, aborted;
+  int32_t mb, mb_it;           // multi-batch execution: phase (PH_*) and poll counter of this context
   unsigned long long sigw;     // last signal word read from this batch's slot
   int32_t out_off, q_off, ovh_n, ovh_t;
   int32_t fwd, nb, count, chain_end;

@@ -90,7 +90,9 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
 }
 
 // Warp 0: output position and queue offset of slot t (exclusive prefix).
-__device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count, int& out_off, int& q_off) {
+// try_only: give up (return true, *ready = 0) after a short poll instead of spinning.
+__device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count, int& out_off, int& q_off,
+                          bool try_only, int* ready) {
   const int lane = threadIdx.x & 31;
   long long sc = 0, sn = 0;
   int j = t - 1;
@@ -132,6 +134,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
       continue;
     }
     j -= __popc(take);
+    if (try_only && it >= 2) { *ready = 0; return true; }
     // after early termination only batches without output may give up (a batch
     // with output precedes the terminating batch, whose look-back saw all of
     // its predecessors' aggregates, so this loop finishes)
@@ -145,6 +148,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
   }
   out_off = (int)(base_out + sc);
   q_off = (int)(base_q + sn);
+  *ready = 1;
   return true;
 }
 
@@ -155,9 +159,14 @@ __device__ __forceinline__ int lb_nb(const KParams& kp, int N, long long V) {
   return N / kp.Bg + (int)(v2 > 1 ? v2 : 1);
 }
 
-// Process one dequeued batch with the look-back chain.
-__device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
-                         uint32_t epoch) {
+// One dequeued batch with the look-back chain, in three phases separated by
+// its two waits (Alg. 5 wait points): lb_phase_a runs up to the
+// Discovered wait, lb_phase_d up to the Counted (prefix) wait, lb_phase_c to
+// the end.  The phases return PH_* (next phase); with try_only a wait that is
+// not yet satisfied returns the same phase (multi-batch execution).
+enum : int32_t { PH_IDLE = 0, PH_CLAIMED = 1, PH_A = 2, PH_D = 3, PH_C = 4, PH_ABORT = 5 };
+
+__device__ __forceinline__ int lb_phase_a(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh) {
   const int t = sh.t, o_begin = sh.o_begin;
   Sig* mine = kp.sig + t;
   clk_mark(kp, sh, 0);
@@ -171,7 +180,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   __syncthreads();
   clk_mark(kp, sh, 1);
   if (oversize) {
-    if (!oversize_discover(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E)) return;
+    if (!oversize_discover(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E)) return PH_ABORT;
   } else {
     discover(kp, P, sm, sh, o_begin, nP, E);
   }
@@ -189,9 +198,8 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
   }
   __syncthreads();
   clk_mark(kp, sh, 3);
-  if (sh.aborted) return;
-  const bool early = sh.s_early == 1;
-  if (early) {
+  if (sh.aborted) return PH_ABORT;
+  if (sh.s_early == 1) {
     trace_ev(kp, t, 3);
     if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
     rediscover_count(kp, P, sm, sh, o_begin, E, true);   // before sorting: removed sort to the end
@@ -204,42 +212,61 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
     clk_mark(kp, sh, 4);
     if (!(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);
     clk_mark(kp, sh, 5);
-  } else {
-    if (!oversize && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // speculative sort
-    clk_mark(kp, sh, 5);
-    beacon(kp, 6, t, 0);
-    if (threadIdx.x < 32) {
-      int ready = 0;
-      if (!lb_wait_discovered(kp, t, false, &ready) && threadIdx.x == 0) sh.aborted = 1;
-    }
-    __syncthreads();
-    clk_mark(kp, sh, 3);
-    if (sh.aborted) return;
-    trace_ev(kp, t, 3);
-    if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
-    if (oversize) {
-      oversize_rediscover_count(kp, P, sm, sh, key0, sm_p_rs(kp)[0], E);
-    } else {
-      rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
-    }
-    if (threadIdx.x == 0) {
-      sh.nb = lb_nb(kp, sh.count, sh.V);
-      st_relaxed_u64(&mine->ovh, lb_pfx(LB_AGG, sh.count, sh.nb));
-      stat_add(kp, &kp.stats->redisc_late, 1);
-    }
-    trace_ev(kp, t, 4);
-    clk_mark(kp, sh, 4);
+    return PH_C;
   }
+  if (!oversize && !(kp.flags & F_NO_SORT)) sort_segments(kp, sm, sh, nP);   // speculative sort
+  clk_mark(kp, sh, 5);
+  beacon(kp, 6, t, 0);
+  return PH_D;
+}
+
+__device__ __forceinline__ int lb_phase_d(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                                          bool try_only) {
+  const int t = sh.t, o_begin = sh.o_begin, E = sh.E;
+  Sig* mine = kp.sig + t;
+  if (threadIdx.x < 32) {
+    int ready = 0;
+    const bool ok = lb_wait_discovered(kp, t, try_only, &ready);
+    if (threadIdx.x == 0) { sh.aborted = ok ? 0 : 1; sh.s_mid = ready; }
+  }
+  __syncthreads();
+  if (sh.aborted) return PH_ABORT;
+  if (!sh.s_mid) return PH_D;
+  clk_mark(kp, sh, 3);
+  trace_ev(kp, t, 3);
+  if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL | LB_DINCL);
+  if (E > kp.T) {
+    oversize_rediscover_count(kp, P, sm, sh, (uint32_t)o_begin + 1, sm_p_rs(kp)[0], E);
+  } else {
+    rediscover_count(kp, P, sm, sh, o_begin, E, true);   // removed: flagged, no re-sort
+  }
+  if (threadIdx.x == 0) {
+    sh.nb = lb_nb(kp, sh.count, sh.V);
+    st_relaxed_u64(&mine->ovh, lb_pfx(LB_AGG, sh.count, sh.nb));
+    stat_add(kp, &kp.stats->redisc_late, 1);
+  }
+  trace_ev(kp, t, 4);
+  clk_mark(kp, sh, 4);
+  return PH_C;
+}
+
+__device__ __forceinline__ int lb_phase_c(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                                          uint32_t epoch, bool try_only) {
+  const int t = sh.t, E = sh.E;
+  const bool oversize = E > kp.T;
+  Sig* mine = kp.sig + t;
   // Counted: prefix over the predecessors' aggregates
   beacon(kp, 8, t, sh.count);
   trace_ev(kp, t, 5);
   if (threadIdx.x < 32) {
-    int out_off = 0, q_off = 0;
-    const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off);
+    int out_off = 0, q_off = 0, ready = 0;
+    const bool ok = lb_prefix(kp, P, t, sh.count, out_off, q_off, try_only, &ready);
     if (threadIdx.x == 0) {
+      sh.s_mid = ready;
       if (!ok) {
         sh.aborted = 1;
-      } else {
+      } else if (ready) {
+        sh.aborted = 0;
         sh.out_off = out_off;
         sh.q_off = q_off;
         if ((long long)q_off + sh.nb > kp.qcap) { latch_error(kp.ctl, ST_CAPACITY); sh.nb = 0; sh.aborted = 1; }
@@ -247,19 +274,22 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
         atomicMax(&kp.ctl->qtail, q_off + sh.nb);
         atomicMax(&kp.ctl->chain_total, out_off + sh.count);
         stat_add(kp, &kp.stats->generated, sh.nb);
+      } else {
+        sh.aborted = 0;
       }
     }
   }
   __syncthreads();
+  if (sh.aborted) return PH_ABORT;
+  if (!sh.s_mid) return PH_C;
   clk_mark(kp, sh, 6);
-  if (sh.aborted) return;
   const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
   beacon(kp, 9, t, out_off);
   trace_ev(kp, t, 6);
   GenState g;
   if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; g.defer = !oversize; }
   if (oversize) {
-    if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) return;
+    if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) return PH_ABORT;
     oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
   } else {
@@ -312,6 +342,106 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
 #endif
   __syncthreads();
   clk_mark(kp, sh, 8);
+  return PH_IDLE;
+}
+
+// Process one dequeued batch with the look-back chain, waiting in place.
+__device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+                                         uint32_t epoch) {
+  int ph = lb_phase_a(kp, P, sm, sh);
+  if (ph == PH_D) ph = lb_phase_d(kp, P, sm, sh, false);
+  if (ph == PH_C) lb_phase_c(kp, P, sm, sh, epoch, false);
+}
+
+// Multi-batch execution: thread 0 polls the claimed slot of a
+// context once.  Returns PH_A (published batch), PH_IDLE (published empty slot,
+// consumed), PH_CLAIMED (not yet published) or PH_ABORT (chain over).
+__device__ int mb_poll(const KParams& kp, ShState& s, uint32_t epoch) {
+  const int t = s.t;
+  if (t >= kp.qcap || ld_relaxed_s32(&kp.ctl->done)) return PH_ABORT;
+  const Desc* d = kp.desc + t;
+  if (ld_relaxed_u32(&d->tag) != epoch) {
+    if ((++s.mb_it & 15) == 0 && lb_chain_exhausted(kp)) return PH_ABORT;
+    return PH_CLAIMED;
+  }
+  (void)ld_acquire_u32(&d->tag);
+  const int b = ld_relaxed_s32(&d->o_begin), e = ld_relaxed_s32(&d->o_end);
+  stat_add(kp, &kp.stats->dequeued, 1);
+  if (b == e) { stat_add(kp, &kp.stats->empty, 1); return PH_IDLE; }
+  trace_ev(kp, t, 0);
+  s.o_begin = b;
+  s.o_end = e;
+  return PH_A;
+}
+
+// Multi-batch execution (RCM_FLAG_MULTI_BATCH, SURVEY.md §8(f) NEXT-2,
+// P:L719-731): every block keeps two batch contexts (own shared scratch and
+// state).  Instead of waiting for Discovered or Counted, the block checks the
+// signal once and moves on to the other context, which may draw a new batch
+// from the queue.  Batches of one block can finish out of order; later ones
+// never overtake earlier ones for Discovered (the look-back enforces it).
+__device__ __noinline__ void chain_worker_mb(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh0, ShState& sh1,
+                                uint32_t epoch) {
+  const uint32_t cbytes = (uint32_t)((smem_bytes(kp.BS, kp.T) + 15) & ~size_t(15));
+  if (threadIdx.x == 0) {
+    sh0.mb = PH_IDLE;
+    sh1.mb = PH_IDLE;
+    for (int i = 0; i < 10; ++i) sh0.clk[i] = sh1.clk[i] = 0;
+    sh0.tclk = sh1.tclk = clock64();
+  }
+  __syncthreads();
+  uint64_t t_idle = 0;   // thread 0: start of the current stretch without progress (watchdog)
+  unsigned ns = 0;
+  for (;;) {
+    bool progress = false;
+    for (int c = 0; c < 2; ++c) {
+      ShState& s = c ? sh1 : sh0;
+      if (threadIdx.x == 0) rcm_ctx_base = c ? cbytes : 0u;
+      __syncthreads();
+      const int ph = s.mb;
+      int nx = ph;
+      if (ph == PH_IDLE) {
+        if (threadIdx.x == 0) {
+          if (ld_relaxed_s32(&kp.ctl->done)) {
+            nx = PH_ABORT;
+          } else {
+            s.t = atomicAdd(&kp.ctl->head, 1);
+            s.mb_it = 0;
+            trace_ev(kp, s.t, 9);
+            nx = PH_CLAIMED;
+          }
+        }
+      } else if (ph == PH_CLAIMED) {
+        if (threadIdx.x == 0) nx = mb_poll(kp, s, epoch);
+      } else if (ph == PH_A) {
+        nx = lb_phase_a(kp, P, sm, s);
+      } else if (ph == PH_D) {
+        nx = lb_phase_d(kp, P, sm, s, true);
+      } else if (ph == PH_C) {
+        nx = lb_phase_c(kp, P, sm, s, epoch, true);
+      }
+      if (threadIdx.x == 0) s.mb = nx;
+      __syncthreads();
+      progress |= s.mb != ph;
+    }
+    if (sh0.mb == PH_ABORT && sh1.mb == PH_ABORT) break;
+    if (threadIdx.x == 0) {
+      if (progress) {
+        t_idle = 0;
+        ns = 0;
+      } else {
+        __nanosleep(ns);
+        if (ns < 128) ns = ns ? ns * 2 : 16;
+        const uint64_t now = globaltimer();
+        if (!t_idle) t_idle = now;
+        else if (now - t_idle > kWatchdogNs) { latch_hang(kp.ctl, 6, sh0.t, sh1.t, sh0.mb * 8 + sh1.mb); }
+      }
+    }
+  }
+  if (threadIdx.x == 0) rcm_ctx_base = 0;
+  if (kp.collect_stats == 2 && threadIdx.x == 0)
+    for (int i = 0; i < 10; ++i) atomicAdd(&kp.stats->stage[i], (unsigned long long)(sh0.clk[i] + sh1.clk[i]));
+  __syncthreads();
 }
 
 __device__ __forceinline__ void chain_worker(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,

@@ -641,7 +641,7 @@ __device__ int block_gl(const KParams& kp, const Problem& P, int32_t* q, int32_t
 // One block orders a whole component (or a whole small matrix, restarting at
 // the C-6 seed when a component is exhausted) with the same batch steps but
 // without the signalling chain: batches are consecutive output ranges.
-__device__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh, int32_t* lev) {
+__device__ __forceinline__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh, int32_t* lev) {
   int seed = P.seed;
   if (P.flags & 2) seed = block_gl(kp, P, kp.o + P.o_base + P.pos0, lev, seed, sh);
   if (threadIdx.x == 0) {

@@ -56,7 +56,7 @@ def test_oracle_and_product_share_no_code():
     pat_prod = re.compile(r"^\s*(import\s+oracle|from\s+oracle|#\s*include\s+.*oracle)", re.M)
     for dirpath, _, files in os.walk(prod):
         for f in files:
-            if f.endswith((".py", ".cu", ".cuh", ".h")):
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 assert not pat_prod.search(open(os.path.join(dirpath, f)).read()), f
     pat_orc = re.compile(r"^\s*(import\s+paper_conf|from\s+paper_conf|#\s*include\s+.*(rcm\.h|csrc))", re.M)
     for f in os.listdir(os.path.join(ROOT, "oracle")):

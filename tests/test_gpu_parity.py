@@ -63,6 +63,8 @@ PATHS = {
     "serial_bs3_noovh": dict(flags=8 | 16 | 1, solo_threshold=-1, batch_nodes=3),
     "serial_noearly": dict(flags=8 | 16 | 2, solo_threshold=-1, batch_nodes=7, temp_elems=2304),
     "leveled": dict(flags=8 | 32, solo_threshold=-1),                # Alg. 2 (NEXT-3)
+    "multi": dict(flags=8 | 64, solo_threshold=-1),                  # multi-batch execution (NEXT-2)
+    "multi_bs3_noearly": dict(flags=8 | 64 | 2, solo_threshold=-1, batch_nodes=3, temp_elems=2304),
 }
 
 
@@ -140,6 +142,15 @@ def test_full_config_parity_leveled(rcm, cfg):
     assert np.array_equal(got, ref)
 
 
+@pytest.mark.parametrize("cfg", [1, 2, 3, 4])
+def test_full_config_parity_multi_batch(rcm, cfg):
+    """NEXT-2: two batches in flight per block -- result-neutral (C-11)."""
+    g, mode, start = synth.config_graph(cfg)
+    ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+    got, _ = _run(rcm, g, mode, start, flags=8 | 64, solo_threshold=-1)
+    assert np.array_equal(got, ref)
+
+
 @pytest.mark.parametrize("cfg", [3, 4])
 def test_full_config_parity_disconnected(rcm, cfg):
     g, mode, start = synth.config_graph(cfg)
@@ -194,7 +205,7 @@ def test_host_argument_errors(rcm):
     plan.close()
 
 
-@pytest.mark.parametrize("opts", [dict(), dict(batch_nodes=64), dict(flags=16)])
+@pytest.mark.parametrize("opts", [dict(), dict(batch_nodes=64), dict(flags=16), dict(flags=64)])
 def test_stress_no_stall_and_determinism(rcm, opts):
     """Repeated runs on one plan: early termination races (a worker abandoning an
     unpublished slot while others are mid look-back) must never stall; every
