@@ -12,6 +12,6 @@ timeout 900 python bench.py --config 5 --steps 5 --warmup 3 > gpurun_out/bench_c
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/ref_c2.json 2> gpurun_out/ref_c2.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/c2_launches.csv python bench.py --config 2 --steps 2 --warmup 3 > gpurun_out/c2_ncu_bench.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_main -s 1 -c 1 -o gpurun_out/prof_c2 python tools/profile_run.py 2 2 > gpurun_out/ncu_c2.log 2>&1
-for lib in base dq128 lb64 slow; do
+for lib in base; do
   RCM_LIB=build/librcm_$lib.so timeout 300 python tools/sweep.py 2 '[{}]' 9 > gpurun_out/sw13_${lib}_c2.jsonl 2> gpurun_out/sw13_${lib}_c2.err
 done
