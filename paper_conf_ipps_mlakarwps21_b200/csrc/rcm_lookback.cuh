@@ -64,7 +64,6 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
     }
     j -= __ffs(~loc & need) - 1;   // verified-LOCAL slots stay LOCAL (monotone)
     if (lane == 0 && (it & 63) == 63) { volatile int32_t* d = kp.dbg + blockIdx.x * 8; d[4] = j; d[5] = (int)a; d[6] = it; }
-    if (try_only && it >= 2) { *ready = 0; return true; }
     // A batch still waiting for Discovered has no aggregate yet, so it is a
     // successor of the batch that completed the order (which saw every
     // predecessor's aggregate): after early termination it has nothing to
@@ -79,6 +78,9 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
       else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 2, t, j, (long long)a); quit = 1; }
     }
     if (__shfl_sync(0xffffffffu, quit, 0)) return false;
+    // try mode gives up only after the termination check above: a batch that
+    // must be abandoned is, even when it is only polled
+    if (try_only && it >= 2) { *ready = 0; return true; }
     lb_spin(ns, it);
   }
   // the flags were polled relaxed: one acquire fence orders this block's
@@ -134,7 +136,6 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
       continue;
     }
     j -= __popc(take);
-    if (try_only && it >= 2) { *ready = 0; return true; }
     // after early termination only batches without output may give up (a batch
     // with output precedes the terminating batch, whose look-back saw all of
     // its predecessors' aggregates, so this loop finishes)
@@ -144,6 +145,7 @@ __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count,
       else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 3, t, j, (long long)b); quit = 1; }
     }
     if (__shfl_sync(0xffffffffu, quit, 0)) return false;   // warp-uniform exit
+    if (try_only && it >= 2) { *ready = 0; return true; }  // after the termination check
     lb_spin(ns, it);
   }
   out_off = (int)(base_out + sc);
@@ -190,11 +192,12 @@ __device__ __forceinline__ int lb_phase_a(const KParams& kp, const Problem& P, c
   // own discovery done: LOCAL.  The release store orders the block's atomicMin
   // marks (performed before discover's closing barrier) ahead of the flag.
   if (threadIdx.x == 0) st_release_u64(&mine->word, LB_LOCAL);
-  // early Discovered: all predecessors already discovered?
-  if (threadIdx.x < 32 && !oversize && !(kp.flags & F_NO_EARLY)) {
+  // early Discovered: all predecessors already discovered?  Warp 1 looks back
+  // while thread 0 (warp 0) waits out the release fence of LOCAL.
+  if (threadIdx.x >= 32 && threadIdx.x < 64 && !oversize && !(kp.flags & F_NO_EARLY)) {
     int ready = 0;
     if (!lb_wait_discovered(kp, t, true, &ready)) ready = -1;
-    if (threadIdx.x == 0) { sh.s_early = ready; if (ready < 0) sh.aborted = 1; }
+    if (threadIdx.x == 32) { sh.s_early = ready; if (ready < 0) sh.aborted = 1; }
   }
   __syncthreads();
   clk_mark(kp, sh, 3);
@@ -423,6 +426,12 @@ __device__ __noinline__ void chain_worker_mb(const KParams& kp, const Problem& P
       if (threadIdx.x == 0) s.mb = nx;
       __syncthreads();
       progress |= s.mb != ph;
+    }
+    if (threadIdx.x == 0) {   // progress beacon of both contexts (rcm_debug_state)
+      volatile int32_t* d = kp.dbg + blockIdx.x * 8;
+      d[4] = sh0.t;
+      d[5] = sh1.t;
+      d[6] = sh0.mb * 8 + sh1.mb;
     }
     if (sh0.mb == PH_ABORT && sh1.mb == PH_ABORT) break;
     if (threadIdx.x == 0) {
