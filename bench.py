@@ -183,6 +183,41 @@ def run_reference_c5(args):
 
 
 # ----------------------------------------------------------------- our arm
+def workload_shape(g, mode, start, ms):
+    """Shape of the traversal the chain must follow: components,
+    the giant component's BFS levels from its RCM seed and its average front
+    (n_component / levels, C-14), Mnodes/s over the giant component only, and the
+    host.  Plain scipy/numpy on the host; not the oracle."""
+    import scipy.sparse as sp
+    from scipy.sparse.csgraph import breadth_first_order, connected_components
+    n = g.n
+    a = sp.csr_matrix((np.ones(g.nnz, dtype=np.int8), g.col_idx, g.row_ptr), shape=(n, n))
+    ncomp, lab = connected_components(a, directed=False)
+    sizes = np.bincount(lab)
+    giant = int(np.argmax(sizes))
+    deg = np.diff(g.row_ptr)
+    members = np.nonzero(lab == giant)[0]
+    if mode == 0 and lab[start] == giant:
+        seed = int(start)
+    else:   # MIN_DEGREE / C-6: min (valence, id) of the component
+        seed = int(members[np.lexsort((members, deg[members]))[0]])
+    order, pred = breadth_first_order(a, seed, directed=False, return_predecessors=True)
+    depth = np.zeros(n, dtype=np.int32)
+    for v in order[1:]:
+        depth[v] = depth[pred[v]] + 1
+    levels = int(depth[order].max()) + 1
+    cpu = ""
+    try:
+        cpu = next(l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name"))
+    except Exception:
+        pass
+    return {"components": int(ncomp), "giant_component_nodes": int(sizes[giant]), "levels_giant": levels,
+            "avg_front_giant": round(int(sizes[giant]) / levels, 1),
+            "giant_mnodes_per_s": round(int(sizes[giant]) / (ms * 1e-3) / 1e6, 3),
+            "us_per_level_giant": round(1e3 * ms / levels, 2),
+            "host_cpu": cpu, "host_cores": os.cpu_count()}
+
+
 def cpu_batch_context(g, mode, start, ref, runs: int = 3):
     """The paper's CPU-BATCH (NEXT-4, libcpubatch.so: Alg. 5 on std::thread) on
     every host core, full workload, median of `runs`: context for the paper's
@@ -338,6 +373,7 @@ def run_ours(args, rank: int, world: int, local_rank: int):
                          "sample": "full workload graph, serial oracle, median of 3 runs"},
         "speedup_vs_oracle": round(o_ms / ms, 2),
         "cpu_batch": cpu_batch_context(g, mode, start, ref) if rank == 0 else None,
+        "workload_shape": workload_shape(g, mode, start, ms) if rank == 0 else None,
         "e2e": {"value": round(e2e_val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 4 * (n + 1) + 4 * nnz,
                 "d2h_bytes_per_step": 4 * n, "ms_per_step": round(e2e_ms / args.steps, 4)},
         "gpu_launches": args.steps,
