@@ -171,6 +171,7 @@ void process_batch(Shared& S, Scratch& W, int32_t t) {
   std::atomic_thread_fence(std::memory_order_release);
   const bool s_mid = me.disc.load(std::memory_order_acquire) == S.tag;   // ln 4
   bool rediscovered = false, counted = false, chain_end = false;
+  const bool early_path = s_early || s_mid;
   int32_t out_off = 0, q_off = 0, nb = 0, count = 0;
   int64_t V = 0;
   auto tally = [&] {
@@ -185,7 +186,6 @@ void process_batch(Shared& S, Scratch& W, int32_t t) {
     forward_discovered(S, t);
     if (!s_early || steal) S.removed.fetch_add(rediscover(S, W, b, np), std::memory_order_relaxed);
     rediscovered = true;
-    S.early.fetch_add(1, std::memory_order_relaxed);
     tally();
     if (me.cnt.load(std::memory_order_acquire) == S.tag) {
       signal_count(S, t, count, V, out_off, q_off, nb, chain_end);
@@ -197,7 +197,6 @@ void process_batch(Shared& S, Scratch& W, int32_t t) {
     if (!wait_tag(S, me.disc)) return;
     forward_discovered(S, t);
     S.removed.fetch_add(rediscover(S, W, b, np), std::memory_order_relaxed);
-    S.late.fetch_add(1, std::memory_order_relaxed);
     tally();
   }
   if (!counted) {   // ln 20-22
@@ -233,6 +232,9 @@ void process_batch(Shared& S, Scratch& W, int32_t t) {
     d.b = d.e = 0;
     d.pub.store(S.tag, std::memory_order_release);
   }
+  // early/late tallied with `executed`, so a batch abandoned at termination
+  // (it returns at a wait above) counts in none of them
+  (early_path ? S.early : S.late).fetch_add(1, std::memory_order_relaxed);
   S.executed.fetch_add(1, std::memory_order_relaxed);
   if (out_off + count == S.n || chain_end) {   // termination
     S.ordered.store(out_off + count);
