@@ -369,7 +369,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   const bool dense = !o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max;
   // dense rows (FEM-like): smaller batches shorten the critical generation
   // chain
-  p->BS = o.batch_nodes ? o.batch_nodes : dense ? 160 : 256;
+  p->BS = o.batch_nodes ? o.batch_nodes : dense ? 192 : 256;
   const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
   const size_t static_sh = 2 * sizeof(ShState) + 64;
   const int nctx = (o.flags & RCM_FLAG_MULTI_BATCH) ? 2 : 1;   // batch contexts per block
@@ -381,6 +381,10 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   if (!T) T = (int)((per_block / nctx - 16 - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
   // dense: B_s rows of ~27 fit; the shared memory left over serves as L1
   if (dense) T = std::min(T, 6144);
+  // sparse rows at the default occupancy: a budget past ~7.7 k candidates buys
+  // few extra parents per batch but takes the SM's L1 (r01d sweep, DESIGN.md §2.1
+  // "batch limits": C3 10.9 -> 9.6 ms, C5 94.7 -> ~70 ms, C4 unchanged)
+  else if (!o.temp_elems && !o.blocks_per_sm && nctx == 1) T = std::min(T, 7680);
   if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;
@@ -518,7 +522,7 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   if (!p->opt.batch_nodes && !p->opt.temp_elems && nnz >= 20ll * n) {
     // dense rows (FEM-like, average valence >= 20) on a plan sized for sparser
     // graphs: cut smaller batches
-    kp.Bg = std::min(kp.BS, 160);
+    kp.Bg = std::min(kp.BS, 192);
     kp.Tg = std::min(kp.T, 6144);
   }
   MainArgs a = make_args(p);
