@@ -200,14 +200,55 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     w.ckey[v] = kKeyMax;
     w.csize[v] = 0;
   }
-  if (gtid() == 0) { w.gctl[1] = 0; w.gctl[2] = 0; }
+  if (gtid() == 0) { w.gctl[1] = 0; w.gctl[2] = 0; w.gctl[3] = -1; }
   grid_barrier(kp);
-  // hook every edge (c < u: the pattern is symmetric) -- thread / warp / block
-  // per row by degree so that hub rows are split across many threads; rows
-  // above 32 entries are listed during the thread pass (front0 / front1)
+  // Sampling (Afforest, Sutton et al. IPDPS'18): hook every unvisited node to
+  // its first kSample unvisited neighbours, so that the giant component is
+  // (mostly) one tree before the full pass.  Its members -- flagged in csize,
+  // a snapshot that stays fixed during the full pass -- then skip their rows;
+  // an edge between a member and a non-member is hooked from the non-member
+  // side, an edge between two members is already inside one tree.
+  constexpr int kSample = 2;
+  for (int u = gtid(); u < n; u += G) {
+    if (ld_cg_s32(w.label + u) < 0) continue;
+    const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
+    int k = 0;
+    for (int e = rs, ee = min(re, rs + 4 * kSample); e < ee && k < kSample; ++e) {   // bounded scan (hub rows)
+      const int c = __ldg(kp.col_idx + e);
+      if (c != u && ld_cg_s32(w.label + c) >= 0) { uf_unite(w.label, u, c); ++k; }
+    }
+  }
+  grid_barrier(kp);
+  if (blockIdx.x == 0) {   // giant = most frequent root among kThreads spread samples
+    int32_t* s_root = reinterpret_cast<int32_t*>(sm_cand(kp));
+    unsigned long long* s_best = reinterpret_cast<unsigned long long*>(s_root + kThreads);
+    const int v = (int)(((long long)threadIdx.x * n) / kThreads);
+    const int r = ld_cg_s32(w.label + v) >= 0 ? uf_find(w.label, v) : -1;
+    s_root[threadIdx.x] = r;
+    if (threadIdx.x == 0) *s_best = 0;
+    __syncthreads();
+    int cnt = 0;
+    for (int i = 0; i < kThreads; ++i) cnt += s_root[i] == r;
+    if (r >= 0) atomicMax(s_best, ((unsigned long long)cnt << 32) | (uint32_t)r);
+    __syncthreads();
+    if (threadIdx.x == 0 && *s_best) w.gctl[3] = (int)(uint32_t)*s_best;
+  }
+  grid_barrier(kp);
+  const int giant = ld_cg_s32(w.gctl + 3);
+  for (int v = gtid(); v < n; v += G) {   // compress + member snapshot
+    if (ld_cg_s32(w.label + v) < 0) continue;
+    const int r = uf_find(w.label, v);
+    w.label[v] = r;
+    w.csize[v] = r == giant;
+  }
+  grid_barrier(kp);
+  // hook every remaining edge (c < u: the pattern is symmetric; or c a member)
+  // -- thread / warp / block per row by degree so that hub rows are split
+  // across many threads; rows above 32 entries are listed during the thread
+  // pass (front0 / front1)
   for (int u = gtid(); u < n; u += G) {
     const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
-    if (ld_cg_s32(w.label + u) < 0) continue;
+    if (ld_cg_s32(w.label + u) < 0 || __ldcg(w.csize + u)) continue;
     if (re - rs > 32) {
       if (re - rs > 4096) w.front1[atomicAdd(w.gctl + 2, 1)] = u;
       else w.front0[atomicAdd(w.gctl + 1, 1)] = u;
@@ -215,7 +256,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     }
     for (int e = rs; e < re; ++e) {
       const int c = __ldg(kp.col_idx + e);
-      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
+      if ((c < u || __ldcg(w.csize + c)) && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
     }
   }
   grid_barrier(kp);
@@ -225,7 +266,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
     for (int e = rs + lane; e < re; e += 32) {
       const int c = __ldg(kp.col_idx + e);
-      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
+      if ((c < u || __ldcg(w.csize + c)) && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
     }
   }
   for (int i = blockIdx.x; i < nbig; i += kp.nblocks) {
@@ -233,9 +274,11 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
     const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
     for (int e = rs + threadIdx.x; e < re; e += kThreads) {
       const int c = __ldg(kp.col_idx + e);
-      if (c < u && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
+      if ((c < u || __ldcg(w.csize + c)) && ld_cg_s32(w.label + c) >= 0) uf_unite(w.label, u, c);
     }
   }
+  grid_barrier(kp);
+  for (int v = gtid(); v < n; v += G) w.csize[v] = 0;   // member flags -> sizes
   grid_barrier(kp);
   // compress; per root: minimum (valence, id) member and size
   // warp-aggregated per root: the giant component's nodes would otherwise all

@@ -271,3 +271,25 @@ def test_disconnected_pseudo_peripheral(rcm):
     for opts in [dict(), dict(solo_threshold=-1, flags=8), dict(solo_threshold=8, flags=8)]:
         got, _ = _run(rcm, g, oracle.PSEUDO_PERIPHERAL, 0, **opts)
         assert np.array_equal(got, ref), opts
+
+
+def _cc_mixes():
+    """Disconnected graphs for the components phase (a13): a dominant component
+    the sampled union-find skips (a relabelled grid, or a hub star whose row
+    exceeds the block-per-row threshold) next to hubs, cliques, paths and
+    isolated nodes, ids shuffled so members and non-members interleave."""
+    small = [synth.path(1), synth.path(2), synth.path(5), synth.complete(40), synth.star(100),
+             synth.cycle(33), synth.path(1), synth.binary_tree(31)]
+    mixes = [synth.disjoint_union([synth.grid3d_27(20, 20, 20, diag=False), synth.star(5000)] + small),
+             synth.disjoint_union([synth.star(20000), synth.grid2d(30, 30)] + small * 3),
+             synth.disjoint_union(small * 40)]
+    return [synth.relabel(g, synth.randperm(g.n, 70 + i)) for i, g in enumerate(mixes)]
+
+
+@pytest.mark.parametrize("path", ["chain", "serial", "multi", "leveled"])
+def test_components_sampled_union_find(rcm, path):
+    for g in _cc_mixes():
+        for mode, start in ((oracle.MIN_DEGREE, 0), (oracle.FIXED, g.n // 3), (oracle.PSEUDO_PERIPHERAL, 0)):
+            ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+            got, st = _run(rcm, g, mode, start, collect_stats=1, **PATHS[path])
+            assert np.array_equal(got, ref), (path, g.n, mode)
