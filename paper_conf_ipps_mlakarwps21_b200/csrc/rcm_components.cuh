@@ -208,7 +208,10 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   // a snapshot that stays fixed during the full pass -- then skip their rows;
   // an edge between a member and a non-member is hooked from the non-member
   // side, an edge between two members is already inside one tree.
-  constexpr int kSample = 2;
+#ifndef RCM_CC_SAMPLE
+#define RCM_CC_SAMPLE 2
+#endif
+  constexpr int kSample = RCM_CC_SAMPLE;
   for (int u = gtid(); u < n; u += G) {
     if (ld_cg_s32(w.label + u) < 0) continue;
     const int rs = __ldg(kp.row_ptr + u), re = __ldg(kp.row_ptr + u + 1);
