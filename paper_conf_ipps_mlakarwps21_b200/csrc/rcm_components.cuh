@@ -209,7 +209,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
   // an edge between a member and a non-member is hooked from the non-member
   // side, an edge between two members is already inside one tree.
 #ifndef RCM_CC_SAMPLE
-#define RCM_CC_SAMPLE 2
+#define RCM_CC_SAMPLE 4
 #endif
   constexpr int kSample = RCM_CC_SAMPLE;
   for (int u = gtid(); u < n; u += G) {
