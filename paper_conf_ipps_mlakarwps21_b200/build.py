@@ -8,12 +8,17 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librcm.so")
-SOURCES = ["rcm.cu"]
-HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh", "rcm_leveled.cuh"]
+SOURCES = ["rcm.cu", "k_main_inst.cu"]
+HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh",
+           "rcm_leveled.cuh", "rcm_main.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-         "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2", "-cudart", "static", "-shared",
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+FLAGS = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2",
          "-Xptxas", "-warn-spills"]
+# one translation unit per persistent-kernel variant (compiled in parallel):
+# (min blocks per SM, multi-batch execution)
+KMAIN_VARIANTS = [(2, 0), (1, 0), (2, 1), (1, 1)]
+BUILD_DIR = os.path.join(HERE, "..", "build", "obj")
 
 
 def _stale() -> bool:
@@ -26,20 +31,41 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps if os.path.exists(d))
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
-        return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
+def _extra_defines() -> list:
     extra = [f"-DRCM_THREADS={os.environ['RCM_THREADS']}"] if os.environ.get("RCM_THREADS") else []
     if os.environ.get("RCM_DISC_U"):
         extra.append(f"-DRCM_DISC_U={os.environ['RCM_DISC_U']}")
     if os.environ.get("RCM_TRACE"):
         extra.append("-DRCM_TRACE")
-    cmd = [NVCC, *FLAGS, *extra, "-o", tmp, *[os.path.join(CSRC, s) for s in SOURCES]]
+    return extra
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    """nvcc -c of every translation unit in parallel, then one -shared link."""
+    if not force and not _stale():
+        return LIB
+    os.makedirs(BUILD_DIR, exist_ok=True)
+    extra = _extra_defines()
     if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd), file=sys.stderr)
-    subprocess.check_call(cmd)
+        extra = ["-Xptxas=-v", *extra]
+    jobs = [(os.path.join(BUILD_DIR, "rcm.o"), [os.path.join(CSRC, "rcm.cu")])]
+    for bps, mb in KMAIN_VARIANTS:
+        jobs.append((os.path.join(BUILD_DIR, f"k_main_{bps}_{mb}.o"),
+                     [f"-DRCM_KBPS={bps}", f"-DRCM_KMB={mb}", os.path.join(CSRC, "k_main_inst.cu")]))
+    procs = []
+    for obj, args in jobs:
+        cmd = [NVCC, *FLAGS, *extra, "-c", "-o", obj + f".tmp{os.getpid()}", *args]
+        if verbose:
+            print(" ".join(cmd), file=sys.stderr)
+        procs.append((obj, subprocess.Popen(cmd)))
+    bad = [obj for obj, p in procs if p.wait() != 0]
+    if bad:
+        raise subprocess.CalledProcessError(1, f"nvcc failed for {bad}")
+    for obj, _ in procs:
+        os.replace(obj + f".tmp{os.getpid()}", obj)
+    tmp = LIB + f".tmp{os.getpid()}"
+    subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-o", tmp,
+                           *[obj for obj, _ in jobs]])
     os.replace(tmp, LIB)
     return LIB
 

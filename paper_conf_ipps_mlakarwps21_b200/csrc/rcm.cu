@@ -9,263 +9,9 @@
 #include <new>
 
 #include "../../include/rcm.h"
-#include "rcm_lookback.cuh"
 #include "rcm_components.cuh"
-#include "rcm_leveled.cuh"
 
 using namespace rcm;
-
-// ===================================================================== phases
-// a1 -- prologue: valence = row_ptr diff, owner word init, argmin of
-// (valence, id) (C-6 / MIN_DEGREE seed), max valence, optional CSR checks.
-// Four nodes per thread with an int4 row_ptr load and a one-element halo.
-__device__ void prologue_phase(const KParams& kp, const MainArgs& a, ShState& sh) {
-  const int n = a.n;
-  unsigned long long best = kKeyMax;
-  int mx = 0, bad = 0;
-  const int G = gthreads(kp);
-  for (int t = gtid(); t * 4 < n; t += G) {
-    const int v0 = t * 4;
-    int r[5];
-    if (a.vec && v0 + 4 <= n) {
-      int4 q = __ldg(reinterpret_cast<const int4*>(kp.row_ptr + v0));
-      r[0] = q.x; r[1] = q.y; r[2] = q.z; r[3] = q.w;
-      r[4] = __ldg(kp.row_ptr + v0 + 4);
-    } else {
-      for (int j = 0; j < 5; ++j) r[j] = (v0 + j <= n) ? __ldg(kp.row_ptr + v0 + j) : 0;
-    }
-    const int m = min(4, n - v0);
-    unsigned long long w[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      if (j < m) {
-        int d = r[j + 1] - r[j];
-        if (d < 0) { bad = 1; d = 0; }
-        w[j] = ((unsigned long long)kInf << 32) | (uint32_t)d;
-        const unsigned long long k = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)(v0 + j);
-        best = k < best ? k : best;
-        mx = max(mx, d);
-      }
-    }
-    if (m == 4) {
-      reinterpret_cast<ulonglong2*>(kp.word + v0)[0] = make_ulonglong2(w[0], w[1]);
-      reinterpret_cast<ulonglong2*>(kp.word + v0)[1] = make_ulonglong2(w[2], w[3]);
-    } else {
-      for (int j = 0; j < m; ++j) kp.word[v0 + j] = w[j];
-    }
-    if (a.validate) {
-      if (v0 == 0 && r[0] != 0) bad = 1;
-      if (v0 + m == n && (long long)r[m] != a.nnz) bad = 1;
-    }
-  }
-  if (a.validate >= 1) {   // every column index in range
-    for (long long i = gtid(); i < a.nnz; i += G) {
-      const int c = __ldg(kp.col_idx + i);
-      bad |= (c < 0 || c >= n);
-    }
-  }
-  best = warp_min_u64(best);
-  for (int d = 16; d > 0; d >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, d));
-  bad = __any_sync(0xffffffffu, bad);
-  if ((threadIdx.x & 31) == 0) {
-    if (best != kKeyMax) atomicMin(&kp.ctl->minkey, best);
-    if (mx) atomicMax(&kp.ctl->maxdeg, mx);
-    if (bad) atomicCAS(&kp.ctl->status, 0, ST_BAD_CSR);
-  }
-}
-
-// validate == 2: structural symmetry -- for every (u, c) the row of c holds u.
-__device__ void validate_sym_phase(const KParams& kp, int n) {
-  int bad = 0;
-  for (int u = gtid(); u < n; u += gthreads(kp)) {
-    for (int e = __ldg(kp.row_ptr + u); e < __ldg(kp.row_ptr + u + 1); ++e) {
-      const int c = __ldg(kp.col_idx + e);
-      if (c < 0 || c >= n) { bad = 1; continue; }
-      bool found = false;
-      for (int f = __ldg(kp.row_ptr + c); f < __ldg(kp.row_ptr + c + 1) && !found; ++f)
-        found = __ldg(kp.col_idx + f) == u;
-      bad |= !found;
-    }
-  }
-  if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicCAS(&kp.ctl->status, 0, ST_NOT_SYM);
-}
-
-// Batched prologue: per matrix k, local valences and the per-matrix argmin.
-__device__ void prologue_batched_phase(const KParams& kp, const MainArgs& a) {
-  const long long stride = (long long)gthreads(kp);
-  for (long long base = (long long)blockIdx.x * kThreads; base < a.total; base += stride) {
-    const long long g = base + threadIdx.x;   // warp-uniform loop; lanes past the end idle
-    const bool valid = g < a.total;
-    int k = -1;
-    unsigned long long key = kKeyMax;
-    if (valid) {
-      int lo = 0, hi = a.num_mats - 1;         // matrix of g: largest k with node_off[k] <= g
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (__ldg(a.node_off + mid) <= g) lo = mid; else hi = mid - 1;
-      }
-      k = lo;
-      const int v = (int)(g - __ldg(a.node_off + k));
-      const int d = max(__ldg(kp.row_ptr + g + k + 1) - __ldg(kp.row_ptr + g + k), 0);
-      kp.word[g] = ((unsigned long long)kInf << 32) | (uint32_t)d;
-      key = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)v;
-    }
-    // lanes of one matrix are contiguous: a segmented shuffle-down min leaves
-    // the segment minimum in its first lane
-    const unsigned peers = __match_any_sync(0xffffffffu, k);
-    unsigned long long m = key;
-    const int lane = threadIdx.x & 31;
-    for (int off = 1; off < 32; off <<= 1) {
-      const unsigned long long o2 = __shfl_down_sync(0xffffffffu, m, off);
-      const int ko = __shfl_down_sync(0xffffffffu, k, off);
-      if (lane + off < 32 && ko == k && o2 < m) m = o2;
-    }
-    if (valid && lane == __ffs(peers) - 1) atomicMin(a.pm_key + k, m);
-  }
-}
-
-// The scheduling phase: every chain problem in turn on all blocks (grid
-// barrier between chains), then the solo problems, one per block at a time.
-template <bool kMB>
-__device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh,
-                                               ShState& sh2) {
-  const int nchain = ld_cg_s32(&kp.ctl->n_chain);
-  for (int c = 0; c < nchain; ++c) {
-    if (kp.chains[c].flags & 2) {   // PSEUDO_PERIPHERAL component: GL seed first (C-5)
-      const int x = gl_phase(kp, a.w, a.n, kp.chains[c].seed, sh);
-      if (blockIdx.x == 0 && threadIdx.x == 0) const_cast<Problem*>(kp.chains)[c].seed = x;
-      grid_barrier(kp);
-    }
-    if (kp.flags & F_LEVELED) {      // NEXT-3: Alg. 2 level-synchronous traversal
-      const Problem PL = kp.chains[c];
-      leveled_chain(kp, a, PL, sm, sh);
-      continue;
-    }
-    if (blockIdx.x == 0 && threadIdx.x == 0) chain_init(kp, kp.chains[c]);
-    grid_barrier(kp);
-    const uint32_t epoch = ld_acquire_u32(&kp.ctl->epoch);
-    // the problem lives in shared memory: its fields are re-read on use (LDS)
-    // instead of pinning 16 registers across the whole traversal
-    if (threadIdx.x == 0) sh.prob = kp.chains[c];
-    __syncthreads();
-    if constexpr (kMB) chain_worker_mb(kp, sh.prob, sm, sh, sh2, epoch);
-    else chain_worker(kp, sh.prob, sm, sh, epoch);
-    grid_barrier(kp);
-    chain_reset_signals(kp);
-    grid_barrier(kp);
-  }
-  const int nsolo = ld_cg_s32(&kp.ctl->n_solo);
-  for (;;) {
-    if (threadIdx.x == 0) {
-      sh.k = atomicAdd(&kp.ctl->solo_next, 1);
-      if (ld_cg_s32(&kp.ctl->status)) sh.k = nsolo;   // block-uniform exit decision
-    }
-    __syncthreads();
-    const int k = sh.k;
-    __syncthreads();
-    if (k >= nsolo) break;
-    if (threadIdx.x == 0) sh.prob = kp.solos[k];
-    __syncthreads();
-    if (sh.prob.size > 0) run_solo(kp, sh.prob, sm, sh, a.w.lev);
-    __syncthreads();
-  }
-}
-
-// One launch per call: reset -> prologue -> seed / problem set-up ->
-// traversal -> (components -> traversal).  Grid barriers between phases.
-template <int kMinBlocks, bool kMB>
-__global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_constant__ KParams kp, const __grid_constant__ MainArgs a) {
-  __shared__ ShState sh;
-  __shared__ ShState sh2;   // second batch context (multi-batch execution, kMB only)
-  SmemPtrs sm;   // layout accessors sm_*(kp) (rcm_batch.cuh)
-  if (threadIdx.x == 0) rcm_ctx_base = 0;
-  const int G = gthreads(kp);
-  // ---- phase 0: reset the per-call control state
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    Ctl* c = kp.ctl;
-    c->ts[0] = globaltimer();
-    c->ts[5] = c->ts[6] = 0;
-    for (int i = 0; i < 8; ++i) c->dbg[i] = 0;
-    c->minkey = kKeyMax; c->maxdeg = 0; c->status = 0; c->head = 0; c->done = 0; c->chain_total = 0;
-    c->solo_next = 0; c->n_chain = 0; c->n_solo = 0; c->n_comp = 0; c->spill_cursor = 0; c->incomplete = 0;
-    if (kp.collect_stats) *kp.stats = Stats{};
-  }
-  if (a.batched)
-    for (int k = gtid(); k < a.num_mats; k += G) a.pm_key[k] = kKeyMax;
-  if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.gl_only) {
-    const long long nn = a.batched ? a.total : a.n;
-    for (long long v = gtid(); v < nn; v += G) a.w.lev[v] = -1;
-  }
-  grid_barrier(kp);
-  // ---- phase 1: prologue (a1)
-  if (a.batched) prologue_batched_phase(kp, a);
-  else prologue_phase(kp, a, sh);
-  if (!a.batched && a.validate == 2) validate_sym_phase(kp, a.n);
-  grid_barrier(kp);
-  stamp(kp, 1);
-  if (ld_cg_s32(&kp.ctl->status)) return;   // read after a barrier: uniform across blocks
-  if (a.gl_only) {   // rcm_find_pseudo_peripheral
-    const int x = gl_phase(kp, a.w, a.n, a.gl_start, sh);
-    if (gtid() == 0) *a.gl_out = x;
-    stamp(kp, 4);
-    return;
-  }
-  // ---- phase 2: problems
-  const int gl_flag = a.mode == RCM_START_PSEUDO_PERIPHERAL ? 2 : 0;
-  if (a.batched) {
-    // LPT: largest matrices first (solo workers dequeue in this order)
-    for (int k = gtid(); k < a.num_mats; k += G) {
-      const long long sz = a.node_off[k + 1] - a.node_off[k];
-      a.w.keys0[k] = ((unsigned long long)(0xffffffffu - (uint32_t)sz) << 32) | (uint32_t)k;
-      a.w.vals0[k] = k;
-    }
-    if (gtid() == 0) { a.w.sctl[0] = a.num_mats; a.w.sctl[1] = 0; }
-    grid_barrier(kp);
-    radix_sort_phase(kp, a.w, 0, 64, reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
-    const int32_t* order = ld_cg_s32(a.w.sctl + 1) ? a.w.vals1 : a.w.vals0;
-    Problem* solos = const_cast<Problem*>(kp.solos);
-    for (int i = gtid(); i < a.num_mats; i += G) {
-      const int k = __ldcg(order + i);
-      Problem P;
-      P.node_base = a.node_off[k];
-      P.rp_base = a.node_off[k] + k;
-      P.ci_base = a.nnz_off[k];
-      P.o_base = a.node_off[k];
-      P.perm_base = a.node_off[k];
-      P.mat_n = (int)(a.node_off[k + 1] - a.node_off[k]);
-      P.pos0 = 0;
-      P.size = P.mat_n;
-      P.seed = (a.mode == RCM_START_FIXED && a.starts) ? a.starts[k] : (int)(uint32_t)__ldcg(a.pm_key + k);
-      P.flags = 1 | gl_flag;
-      P.pad = 0;
-      solos[i] = P;
-    }
-    if (gtid() == 0) kp.ctl->n_solo = a.num_mats;
-  } else {
-    int seed = a.mode == RCM_START_FIXED ? a.start : (int)(uint32_t)__ldcg(&kp.ctl->minkey);
-    if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.solo) seed = gl_phase(kp, a.w, a.n, seed, sh);
-    if (gtid() == 0) {
-      Problem P;
-      P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
-      P.mat_n = a.n; P.pos0 = 0; P.size = a.n; P.seed = seed; P.pad = 0;
-      if (a.solo) { P.flags = 1 | gl_flag; const_cast<Problem*>(kp.solos)[0] = P; kp.ctl->n_solo = 1; }
-      else { P.flags = 0; const_cast<Problem*>(kp.chains)[0] = P; kp.ctl->n_chain = 1; }
-    }
-  }
-  grid_barrier(kp);
-  stamp(kp, 2);
-  // ---- phase 3: the traversal (a2-a12)
-  schedule_phase<kMB>(kp, a, sm, sh, sh2);
-  grid_barrier(kp);
-  stamp(kp, 3);
-  // ---- phase 4: components left over by the chain-first pass (a13)
-  if (!a.batched && !a.solo && ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
-    cc_phase(kp, a, sm, sh);
-    schedule_phase<kMB>(kp, a, sm, sh, sh2);
-    grid_barrier(kp);
-  }
-  stamp(kp, 4);
-}
 
 // ======================================================================= host
 struct rcm_plan {
@@ -334,16 +80,17 @@ extern "C" void rcm_plan_destroy(rcm_plan_t p) {
   delete p;
 }
 
-// k_main instantiation for `bps` resident blocks per SM (register budget
-// 64K / (bps * kThreads)); capped at 1024 threads per SM (64 registers).
+// k_main instantiations (k_main_inst.cu, one translation unit each): 1 or 2
+// resident blocks per SM (register budget 64K / (bps * kThreads)), with or
+// without multi-batch execution.
+extern "C" const void* rcm_kmain_ptr_1_0();
+extern "C" const void* rcm_kmain_ptr_2_0();
+extern "C" const void* rcm_kmain_ptr_1_1();
+extern "C" const void* rcm_kmain_ptr_2_1();
 static const void* pick_kernel(int bps, bool mb) {
-  constexpr int kMaxBps = 1024 / kThreads;   // >= 64 registers per thread
-  const int b = std::min(bps, kMaxBps);
-  if (mb) return b >= 2 ? (const void*)k_main<(kMaxBps >= 2 ? 2 : 1), true> : (const void*)k_main<1, true>;
-  if (b >= 4) return (const void*)k_main<(kMaxBps >= 4 ? 4 : 1), false>;
-  if (b == 3) return (const void*)k_main<(kMaxBps >= 3 ? 3 : 1), false>;
-  if (b == 2) return (const void*)k_main<(kMaxBps >= 2 ? 2 : 1), false>;
-  return (const void*)k_main<1, false>;
+  static_assert(1024 / kThreads >= 2, "two 512-thread blocks per SM");
+  if (mb) return bps >= 2 ? rcm_kmain_ptr_2_1() : rcm_kmain_ptr_1_1();
+  return bps == 2 ? rcm_kmain_ptr_2_0() : rcm_kmain_ptr_1_0();
 }
 
 extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t nnz_max,

@@ -42,7 +42,7 @@ struct KParams {
 // (5), prefix known (6), output written (7), batches published (8);
 // [kTraceW-1] = generator slot << 32 | block.  Thread 0 only.
 constexpr int kTraceW = 16;
-__device__ __noinline__ void trace_ev_slow(unsigned long long* trace, int cap, int slot, int ev) {
+static __device__ __noinline__ void trace_ev_slow(unsigned long long* trace, int cap, int slot, int ev) {
   if (trace && slot >= 0 && slot < cap) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -165,7 +165,7 @@ __device__ __forceinline__ void send_sig(Sig* s, unsigned long long w) { st_rele
 
 // Busy wait: tight polling first, then sleep back-off.  Returns
 // the signal word, or 0 if the chain was terminated (done) or the watchdog fired.
-__device__ unsigned long long wait_sig(const Sig* s, uint32_t need, Ctl* ctl) {
+static __device__ unsigned long long wait_sig(const Sig* s, uint32_t need, Ctl* ctl) {
   unsigned long long w = load_sig(s);
   if (sig_state(w) >= need) return w;
   uint64_t t0 = 0;
@@ -190,7 +190,7 @@ __device__ unsigned long long wait_sig(const Sig* s, uint32_t need, Ctl* ctl) {
 // exclusive prefix of their row lengths into p_eo.  If cut_T, shrink nP to the
 // longest prefix whose edge count fits T (at least one parent) -- the solo
 // worker's batch formation.  Returns nP; sh.E = edge slots.
-__device__ int load_parents(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+static __device__ int load_parents(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                             int o_begin, int nP, bool cut_T) {
   for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
     int v = ld_cg_s32(kp.o + P.o_base + o_begin + lp);
@@ -248,7 +248,7 @@ __device__ __forceinline__ int find_parent(const int32_t* p_eo, int lo, int nP, 
 // iff the old owner was larger.  The valence comes back in the same 64-bit word
 // ("immediately compute the valence").  Candidates go to p's segment
 // of the scratchpad ("atomicAdd to reserve a unique spot").
-__device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+static __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                          int o_begin, int nP, int E) {
   for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm_p_cnt(kp)[lp] = 0;
   __syncthreads();
@@ -309,7 +309,7 @@ __device__ void discover(const KParams& kp, const Problem& P, const SmemPtrs& sm
 // become kKeyMax.  Then sh.count = kept children and sh.V = the sum of their
 // valences clamped to Tg (oversize valences are clamped, they get
 // their own batch).  One combined block reduction.
-__device__ void rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+static __device__ void rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                                  int o_begin, int E, bool check) {
   const unsigned long long* word = kp.word + P.node_base;
   long long kr = 0, val = 0;   // kept << 32 | removed, clamped valence sum
@@ -400,7 +400,7 @@ __device__ __forceinline__ void bitonic_sort_flip(unsigned long long* a, int n, 
 // (valence, id) -- Alg. 1 ln 14 "sort(c)" per parent, equivalently the
 // GPU key (local parent, valence) of P:L778-781 with the id tie-break of C-1.
 // Tiny segments: one thread (insertion sort); medium: one warp; large: block.
-__device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh, int nP) {
+static __device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh, int nP) {
   if (threadIdx.x == 0) sh.big_n = 0;
   __syncthreads();
   for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
@@ -463,7 +463,7 @@ __device__ void sort_segments(const KParams& kp, const SmemPtrs& sm, ShState& sh
 // of (kept << 40 | clamped valence) over contiguous per-thread chunks gives
 // the positions; with `gen` the scan is also left in cand[0..E] for batch
 // generation (gen_chunk): cand[i] = exclusive prefix of slot i, cand[E] = total.
-__device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+static __device__ void write_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                              int E, int out_off, bool gen) {
   const int per = (E + kThreads - 1) / kThreads;
   const int b = threadIdx.x * per, e = min(E, b + per);
@@ -551,7 +551,7 @@ __device__ __forceinline__ void gen_close(const KParams& kp, GenState& g, int en
 // Consume one chunk of ordered nodes.  pre[i] (i <= m) = exclusive prefix over
 // the chunk's slots of (count << 40 | clamped valence); slot i's node sits at
 // matrix-local position base + (pre[i] >> 40).  Thread 0 only.
-__device__ void gen_chunk(const KParams& kp, GenState& g, const unsigned long long* pre, int m,
+static __device__ void gen_chunk(const KParams& kp, GenState& g, const unsigned long long* pre, int m,
                           int base, int q_off, int nb, uint32_t epoch) {
   const unsigned long long kMaskV = (1ull << 40) - 1;
   int a = 0;   // first slot not yet assigned
@@ -585,7 +585,7 @@ __device__ void gen_chunk(const KParams& kp, GenState& g, const unsigned long lo
   }
 }
 
-__device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, int nb,
+static __device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, int nb,
                            uint32_t epoch) {
   if (g.cnt > 0) gen_close(kp, g, end, q_off, nb, epoch);
   if (g.has_pend) {
@@ -597,7 +597,7 @@ __device__ void gen_finish(const KParams& kp, GenState& g, int end, int q_off, i
 }
 
 // Publish empty batches q_off + [from, nb) (all threads of warp 0).
-__device__ void publish_empties(const KParams& kp, int q_off, int from, int nb, uint32_t epoch) {
+static __device__ void publish_empties(const KParams& kp, int q_off, int from, int nb, uint32_t epoch) {
   if (threadIdx.x < 32) {
     for (int i = from + threadIdx.x; i < nb; i += 32) publish_desc(kp.desc + q_off + i, 0, 0, q_off + i + 1, epoch);
   }

@@ -71,7 +71,7 @@ __device__ __forceinline__ void stamp(const KParams& kp, int i) {
 // (8-bit digits; the order of equal keys -- and thus of bits below lo_bit when
 // the input is already ordered by them -- is preserved).  Count in w.sctl[0]; w.sctl[1] = buffer holding the data.
 // A digit that is equal in all keys is skipped.  `scratch`: >= 17 KB smem.
-__device__ void radix_sort_phase(const KParams& kp, const CompWS& w, int lo_bit, int hi_bit, int32_t* scratch,
+static __device__ void radix_sort_phase(const KParams& kp, const CompWS& w, int lo_bit, int hi_bit, int32_t* scratch,
                                  ShState& sh) {
   const int count = ld_cg_s32(w.sctl);
   if (count <= 1) return;
@@ -187,7 +187,7 @@ __device__ __forceinline__ void chunk_of(const KParams& kp, long long n, long lo
   e = min(n, b + C);
 }
 
-__device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
+static __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh) {
   const CompWS& w = a.w;
   const int n = a.n;
   const int G = gthreads(kp);
@@ -433,7 +433,7 @@ __device__ void cc_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& s
 // P:L365-375 with reading C-5: BFS from r; x = min (valence, id) node of the
 // last level; BFS from x; continue while the level count grows; return x.
 // Level-synchronous BFS, frontier queues in HBM, grid barrier per level.
-__device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
+static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
   const int G = gthreads(kp);
   for (int v = gtid(); v < n; v += G) w.lev[v] = -1;
   grid_barrier(kp);
@@ -478,7 +478,7 @@ __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, ShState&
   return level + 1;
 }
 
-__device__ int gl_phase(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
+static __device__ int gl_phase(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
   int nl = gl_bfs(kp, w, n, r, sh);
   for (;;) {
     const int x = (int)(uint32_t)__ldcg(w.gkey);

@@ -15,7 +15,7 @@
 
 namespace rcm {
 
-__device__ void leveled_chain(const KParams& kp, const MainArgs& a, const Problem& P, const SmemPtrs& sm,
+static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const Problem& P, const SmemPtrs& sm,
                               ShState& sh) {
   const CompWS& w = a.w;
   const int G = gthreads(kp);

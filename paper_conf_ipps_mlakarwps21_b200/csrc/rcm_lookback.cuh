@@ -45,7 +45,7 @@ __device__ __forceinline__ void lb_spin(unsigned& ns, int it) {
 
 // Warp 0: wait until every slot < t is discovered.  Returns false on error.
 // try_only: give up (return false, *ready = 0) instead of spinning.
-__device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int* ready) {
+static __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int* ready) {
   const int lane = threadIdx.x & 31;
   int j = t - 1;
   unsigned ns = 0;
@@ -93,7 +93,7 @@ __device__ bool lb_wait_discovered(const KParams& kp, int t, bool try_only, int*
 
 // Warp 0: output position and queue offset of slot t (exclusive prefix).
 // try_only: give up (return true, *ready = 0) after a short poll instead of spinning.
-__device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count, int& out_off, int& q_off,
+static __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int count, int& out_off, int& q_off,
                           bool try_only, int* ready) {
   const int lane = threadIdx.x & 31;
   long long sc = 0, sn = 0;
@@ -359,7 +359,7 @@ __device__ __forceinline__ void lb_batch(const KParams& kp, const Problem& P, co
 // Multi-batch execution: thread 0 polls the claimed slot of a
 // context once.  Returns PH_A (published batch), PH_IDLE (published empty slot,
 // consumed), PH_CLAIMED (not yet published) or PH_ABORT (chain over).
-__device__ int mb_poll(const KParams& kp, ShState& s, uint32_t epoch) {
+static __device__ int mb_poll(const KParams& kp, ShState& s, uint32_t epoch) {
   const int t = s.t;
   if (t >= kp.qcap || ld_relaxed_s32(&kp.ctl->done)) return PH_ABORT;
   const Desc* d = kp.desc + t;
@@ -383,7 +383,7 @@ __device__ int mb_poll(const KParams& kp, ShState& s, uint32_t epoch) {
 // signal once and moves on to the other context, which may draw a new batch
 // from the queue.  Batches of one block can finish out of order; later ones
 // never overtake earlier ones for Discovered (the look-back enforces it).
-__device__ __noinline__ void chain_worker_mb(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh0, ShState& sh1,
+static __device__ __noinline__ void chain_worker_mb(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh0, ShState& sh1,
                                 uint32_t epoch) {
   const uint32_t cbytes = (uint32_t)((smem_bytes(kp.BS, kp.T) + 15) & ~size_t(15));
   if (threadIdx.x == 0) {

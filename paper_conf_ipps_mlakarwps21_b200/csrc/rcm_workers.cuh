@@ -13,7 +13,7 @@ __device__ __forceinline__ void stat_add(const KParams& kp, unsigned long long* 
 
 // Seed a component: o[pos] = s, perm[N-1-pos] = s, owner(s) = 0 (the root key,
 // smaller than every parent key pos+1).  Thread 0 only.
-__device__ void place_root(const KParams& kp, const Problem& P, int s, int pos) {
+static __device__ void place_root(const KParams& kp, const Problem& P, int s, int pos) {
   kp.o[P.o_base + pos] = s;
   kp.perm[P.perm_base + P.mat_n - 1 - pos] = s;
   if (kp.iperm) kp.iperm[P.node_base + s] = P.mat_n - 1 - pos;
@@ -22,7 +22,7 @@ __device__ void place_root(const KParams& kp, const Problem& P, int s, int pos) 
   atomicMin(wp, w & 0xffffffffull);
 }
 
-__device__ void grid_barrier(const KParams& kp) {
+static __device__ void grid_barrier(const KParams& kp) {
   beacon(kp, 11, -1, ld_relaxed_s32(&kp.ctl->gbar_gen));
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -45,7 +45,7 @@ __device__ void grid_barrier(const KParams& kp) {
 }
 
 // Unvisited node of minimum (valence, id) of a matrix (C-6), or -1.
-__device__ int block_argmin_unvisited(const KParams& kp, const Problem& P, ShState& sh) {
+static __device__ int block_argmin_unvisited(const KParams& kp, const Problem& P, ShState& sh) {
   unsigned long long best = kKeyMax;
   const unsigned long long* word = kp.word + P.node_base;
   for (int v = threadIdx.x; v < P.mat_n; v += kThreads) {
@@ -73,7 +73,7 @@ __device__ int block_argmin_unvisited(const KParams& kp, const Problem& P, ShSta
 // Stable LSD radix sort (8-bit digits) of a[0..n) in global memory by one
 // block, temp buffer tmp[0..n); digits that are equal in all keys are skipped.
 // `scratch` is >= (1 + kWarps) * 256 ints of shared memory.
-__device__ void block_radix_sort_global(unsigned long long* a, unsigned long long* tmp, int n,
+static __device__ void block_radix_sort_global(unsigned long long* a, unsigned long long* tmp, int n,
                                         int32_t* scratch, ShState& sh) {
   if (n <= 1) return;
   unsigned long long first = __ldcg(a);
@@ -152,7 +152,7 @@ __device__ void block_radix_sort_global(unsigned long long* a, unsigned long lon
 // claims are kept in a shared-memory bitmap over the row; after rediscovery the
 // kept children are gathered into plan-owned HBM scratch, sorted by
 // (valence, id) there, written out, and cut into batches chunk by chunk.
-__device__ bool oversize_discover(const KParams& kp, const Problem& P, const SmemPtrs& sm,
+static __device__ bool oversize_discover(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                   ShState& sh, uint32_t key, int rs, int D) {
   uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
@@ -183,7 +183,7 @@ __device__ bool oversize_discover(const KParams& kp, const Problem& P, const Sme
 }
 
 // Rediscover (keep iff owner == key), then count and clamped valence sum.
-__device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm,
+static __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                           ShState& sh, uint32_t key, int rs, int D) {
   uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
@@ -215,7 +215,7 @@ __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, c
 }
 
 // Gather kept children into spill, sort them.  Returns false on capacity error.
-__device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const SmemPtrs& sm,
+static __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                      ShState& sh, int rs, int D) {
   uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
@@ -257,7 +257,7 @@ __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const 
 
 // Write the sorted children at out_off and cut them into batches.
 // Thread-0 generation state g must be initialised by the caller (overhang).
-__device__ void oversize_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
+static __device__ void oversize_output(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh,
                                 int out_off, bool generate, GenState& g, int q_off, int nb,
                                 uint32_t epoch) {
   const int C = sh.count;
@@ -303,7 +303,7 @@ __device__ void oversize_output(const KParams& kp, const Problem& P, const SmemP
 // and the predecessor's output position received (signal word `w`), forward the
 // position, the queue offset and possibly an overhang to the successor.
 // Thread 0 only.
-__device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, unsigned long long w,
+static __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, unsigned long long w,
                              Sig* succ_sig, int succ) {
   const int out_off = sig_out(w);
   const int q_off = sig_q(w);
@@ -358,7 +358,7 @@ __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* mine, un
 // reservation raised `qtail` (release), and every reserved slot is counted
 // exactly once, so completed == qtail read in this order (acquire) implies no
 // slot is still running.  Polled by blocks idling in dequeue.
-__device__ __noinline__ bool lb_chain_exhausted(const KParams& kp) {
+static __device__ __noinline__ bool lb_chain_exhausted(const KParams& kp) {
   const int c = ld_acquire_s32(&kp.ctl->completed);
   if (c != ld_acquire_s32(&kp.ctl->qtail)) return false;
   kp.ctl->incomplete = 1;   // idempotent: several idle blocks may get here
@@ -368,7 +368,7 @@ __device__ __noinline__ bool lb_chain_exhausted(const KParams& kp) {
 }
 
 // Thread 0; returns false when the chain is done.
-__device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
+static __device__ bool dequeue(const KParams& kp, ShState& sh, uint32_t epoch) {
   for (;;) {
     if (ld_relaxed_s32(&kp.ctl->done)) return false;
     const int t = atomicAdd(&kp.ctl->head, 1);
@@ -545,7 +545,7 @@ __device__ __forceinline__ void chain_batch(const KParams& kp, const Problem& P,
 // Chain set-up (a2): slot 0 = the seed batch [pos0, pos0+1) whose virtual
 // predecessor is Completed with out_off = pos0+1 and queue tail 1.  Thread 0 of
 // block 0, before a grid barrier.
-__device__ void chain_init(const KParams& kp, const Problem& P) {
+static __device__ void chain_init(const KParams& kp, const Problem& P) {
   const uint32_t ep = atomicAdd(&kp.ctl->epoch, 1u) + 1u;
   kp.ctl->head = 0;
   kp.ctl->done = 0;
@@ -567,7 +567,7 @@ __device__ void chain_init(const KParams& kp, const Problem& P) {
 
 // After a chain run (all blocks, between grid barriers): zero the signal slots
 // it used so the next run starts from S_NONE without an epoch in the word.
-__device__ void chain_reset_signals(const KParams& kp) {
+static __device__ void chain_reset_signals(const KParams& kp) {
   const int qt = min(ld_cg_s32(&kp.ctl->qtail) + 2, kp.qcap + 1);
   for (int i = blockIdx.x * kThreads + threadIdx.x; i < qt; i += kp.nblocks * kThreads) {
     kp.sig[i].word = 0;
@@ -580,7 +580,7 @@ __device__ void chain_reset_signals(const KParams& kp) {
 // (P:L365-375): the queue lives in the component's still-unwritten output
 // range q[], levels in lev[] (-1 = unvisited; reset before returning).
 // Returns the number of levels; sh.minkey = min (valence, id) of the last level.
-__device__ int block_bfs(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
+static __device__ int block_bfs(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
   int32_t* lv = lev + P.node_base;
   const int32_t* rp = kp.row_ptr + P.rp_base;
   const int32_t* col = kp.col_idx + P.ci_base;
@@ -625,7 +625,7 @@ __device__ int block_bfs(const KParams& kp, const Problem& P, int32_t* q, int32_
 }
 
 // GL finder (C-5) from r inside its component, block-level.
-__device__ int block_gl(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
+static __device__ int block_gl(const KParams& kp, const Problem& P, int32_t* q, int32_t* lev, int r, ShState& sh) {
   int nl = block_bfs(kp, P, q, lev, r, sh);
   int x = (int)(uint32_t)sh.minkey;
   __syncthreads();
