@@ -1,19 +1,23 @@
 #!/usr/bin/env python
 """Benchmark of the batch-RCM hot path (one JSON line on rank 0).
 
-Workload (default, BASELINE.json configs[1]): C2 = 3D 27-point FEM-like grid
-100^3 (1,000,000 nodes, 26,463,592 nnz), diagonal stored, random relabel
-(seed 2), MIN_DEGREE start -- see DESIGN.md "Input recipe".  A step = one
-rcm_reorder call (prologue + traversal + fused reverse) on device-resident
-input; the L2 is flushed before every timed step (input ~110 MB < 126 MB L2).
+Headline workload (default, the largest single-GPU configuration and the only
+one that shards): C5 = the batch of 8,192 independent 2D 5-point / 3D 27-point
+mesh matrices, 1k-100k nodes each (~176 M nodes, ~2.67 G nnz), diagonal stored,
+per-matrix random relabel, MIN_DEGREE start per matrix -- DESIGN.md "Input
+recipe".  A step = one rcm_reorder_batched call (all 8,192 matrices) on
+device-resident input (11 GB, larger than the 126 MB L2); with N > 1 GPUs the
+matrices are sharded (LPT on nnz) and the step includes the NCCL gather of the
+permutations into rank 0.  C4 (R-MAT 2^22, one graph) and C2 (27-point grid
+100^3) are reported in the same line under "secondary" (N = 1 only).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--config 2|5]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--config 1..5]
 
-N > 1 (torchrun): C1-C4 are one connected graph each and stay on one GPU, so
-every rank reorders its own replica ("replicas only"); config 5
-shards independent matrices across ranks and gathers the permutations with
-NCCL.  --impl reference times the serial oracle (the deliberately slow
-baseline) on the host cores of rank 0.
+--gpus N without torchrun re-launches itself under torch.distributed.run with N
+ranks.  C1-C4 with N > 1 are replicas (each rank orders its own copy; a
+connected graph stays on one GPU): value = n / max-over-ranks time, no
+speed-up claimed.  --impl reference times the serial oracle (the deliberately
+slow baseline) on rank 0's host cores on a bounded sample of the same workload.
 """
 from __future__ import annotations
 
@@ -24,7 +28,6 @@ import statistics
 import subprocess
 import sys
 import tempfile
-import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -33,14 +36,34 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 HBM_FALLBACK_GBS = 6650.0
+METRIC_FALLBACK = "RCM Mnodes/s and ms/matrix vs host serial RCM; % of HBM roofline"
+
+
+def _metric() -> str:
+    """BASELINE.json's metric string, verbatim (both arms print the same one)."""
+    try:
+        return json.load(open(os.path.join(ROOT, "BASELINE.json")))["metric"]
+    except Exception:
+        return METRIC_FALLBACK
 
 
 def _peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
         d = json.load(open(p))
-        return float(d["hbm_gbs"]), "measured"
-    return HBM_FALLBACK_GBS, "fallback"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    return HBM_FALLBACK_GBS, "fallback (B200_PROFILING.md)"
+
+
+def _cores() -> int:
+    return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+
+
+def _cpu_model() -> str:
+    try:
+        return next(l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name"))
+    except Exception:
+        return ""
 
 
 # ------------------------------------------------------------------ clocks
@@ -58,7 +81,7 @@ class ClockSampler:
         try:
             self.f = tempfile.NamedTemporaryFile("w+", delete=False, suffix=".csv")
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.proc = None
@@ -66,7 +89,7 @@ class ClockSampler:
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
-        time.sleep(0.25)
+        time.sleep(0.15)
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -90,26 +113,8 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-# ----------------------------------------------------------------- inputs
-def load_workload(cfg: int):
-    import synth
-    if cfg in (1, 2, 3, 4):
-        g, mode, start = synth.config_graph(cfg)
-        names = {1: "C1 2D 5-point Laplacian 64x64, shuffled labels, FIXED start 0",
-                 2: "C2 3D 27-point FEM-like grid 100^3, random relabel, MIN_DEGREE start",
-                 3: "C3 random geometric graph 4M nodes, mean degree 14, MIN_DEGREE start",
-                 4: "C4 R-MAT 2^22 (0.57,0.19,0.19,0.05) x 8 edge samples, MIN_DEGREE start"}
-        return g, mode, start, names[cfg]
-    raise ValueError(cfg)
-
-
-def _plan_env() -> dict:
-    """Plan options from RCM_PLAN (JSON), for tuning sweeps; empty by default."""
-    return json.loads(os.environ["RCM_PLAN"]) if os.environ.get("RCM_PLAN") else {}
-
-
-def traffic_from_profile(cfg: int):
-    p = os.path.join(ROOT, "profiles", f"traffic_c{cfg}.json")
+def traffic_from_profile(key: str):
+    p = os.path.join(ROOT, "profiles", f"traffic_{key}.json")
     if os.path.exists(p):
         try:
             return json.load(open(p)).get("dram_bytes_per_launch")
@@ -118,139 +123,130 @@ def traffic_from_profile(cfg: int):
     return None
 
 
+def _plan_env() -> dict:
+    """Plan options from RCM_PLAN (JSON), for tuning sweeps; empty by default."""
+    return json.loads(os.environ["RCM_PLAN"]) if os.environ.get("RCM_PLAN") else {}
+
+
+CONFIG_NAMES = {
+    1: "C1 2D 5-point Laplacian 64x64, shuffled labels, FIXED start 0",
+    2: "C2 3D 27-point FEM-like grid 100^3, random relabel, MIN_DEGREE start",
+    3: "C3 random geometric graph 4M nodes, mean degree 14, MIN_DEGREE start",
+    4: "C4 R-MAT 2^22 (0.57,0.19,0.19,0.05) x 8 edge samples, MIN_DEGREE start",
+    5: "C5 batch of 8192 2D 5-point / 3D 27-point mesh matrices (1k-100k nodes), MIN_DEGREE per matrix",
+}
+
+
+def c5_sample(num, count, seed=12345):
+    """Seeded sample of config-5 matrices (largest, smallest, random)."""
+    import synth
+    sizes = synth.c5_sizes(num)
+    rng = np.random.default_rng(seed)
+    pick = {int(np.argmax(sizes)), int(np.argmin(sizes))}
+    pick.update(int(k) for k in rng.choice(num, min(count, num), replace=False))
+    return sorted(pick)
+
+
 # ------------------------------------------------------------ reference arm
 def run_reference(args, rank: int):
+    """The serial oracle as it stands (oracle/, plain C, one matrix per thread
+    for the batch) on rank 0's host cores, on a bounded seeded sample of the
+    workload per step.  Other ranks exit without work."""
     if rank != 0:
         return
     import oracle
-    if args.config == 5:
-        return run_reference_c5(args)
-    g, mode, start, name = load_workload(args.config)
-    oracle.build()
-    for _ in range(args.warmup):
-        oracle.rcm(g.row_ptr, g.col_idx, mode, start)
-    ts = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        oracle.rcm(g.row_ptr, g.col_idx, mode, start)
-        ts.append(time.perf_counter() - t0)
-    ms = 1e3 * sum(ts) / len(ts)
-    val = g.n / (ms * 1e-3) / 1e6
-    line = {
-        "impl": "reference", "metric": "RCM Mnodes/s (serial oracle, host)", "value": round(val, 3),
-        "unit": "Mnodes/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": round(ms, 4), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "i32", "data": "synthetic",
-        "config": {"workload": name, "n": g.n, "nnz": g.nnz},
-        "cpu_baseline": {"value": round(val, 3), "unit": "Mnodes/s", "cores": 1, "kind": "oracle",
-                         "sample": f"full workload graph, {args.steps} timed runs of the serial oracle"},
-        "e2e": {"value": round(val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-    }
-    print(json.dumps(line), flush=True)
-
-
-def run_reference_c5(args):
-    """Serial oracle on a bounded, seeded sample of the config-5 matrices per step."""
-    import oracle
     import synth
     oracle.build()
-    sizes = synth.c5_sizes(args.num_mats)
-    sample = c5_sample(args.num_mats, 6)
-    mats = {k: synth.c5_matrix(k, int(sizes[k])) for k in sample}
+    cores = _cores()
+    if args.config == 5:
+        sizes = synth.c5_sizes(args.num_mats)
+        sample = c5_sample(args.num_mats, 256)
+        b = synth.batch_of([synth.c5_matrix(k, int(sizes[k])) for k in sample])
+        nodes = int(b.node_off[-1])
+
+        def one():
+            oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, oracle.MIN_DEGREE,
+                               threads=cores)
+        desc = (f"{len(sample)} of {args.num_mats} config-5 matrices ({nodes} nodes) per step, "
+                f"independent matrices on a {cores}-thread pool")
+        mats = len(sample)
+    else:
+        g, mode, start = synth.config_graph(args.config)
+        nodes = g.n
+        mats = 1
+
+        def one():
+            oracle.rcm(g.row_ptr, g.col_idx, mode, start)
+        desc = "the full workload graph per step, one core (RCM is serial, P:L65-66)"
+        cores = 1
     for _ in range(args.warmup):
-        for g in mats.values():
-            oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE)
-    nodes = sum(g.n for g in mats.values())
+        one()
     ts = []
     for _ in range(args.steps):
         t0 = time.perf_counter()
-        for g in mats.values():
-            oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE)
+        one()
         ts.append(time.perf_counter() - t0)
-    sec = sum(ts) / len(ts)
+    sec = statistics.mean(ts)
     val = nodes / sec / 1e6
     print(json.dumps({
-        "impl": "reference", "metric": "RCM Mnodes/s (serial oracle, host)", "value": round(val, 3),
-        "unit": "Mnodes/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": round(1e3 * sec, 4), "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-        "dtype": "i32", "data": "synthetic",
-        "config": {"workload": f"C5 batch of {args.num_mats} mesh matrices (bounded sample per step)",
-                   "sample_matrices": sample, "sample_nodes": nodes},
-        "cpu_baseline": {"value": round(val, 3), "unit": "Mnodes/s", "cores": 1, "kind": "oracle",
-                         "sample": f"{len(sample)} matrices ({nodes} nodes) per step"},
+        "impl": "reference", "metric": _metric(), "value": round(val, 3), "unit": "Mnodes/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * sec, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "i32", "data": "synthetic",
+        "config": {"workload": CONFIG_NAMES[args.config], "sample_nodes": nodes, "sample_matrices": mats,
+                   "ms_per_matrix": round(1e3 * sec / mats, 6)},
+        "cpu_baseline": {"value": round(val, 3), "unit": "Mnodes/s", "cores": cores, "kind": "oracle",
+                         "sample": desc, "host_cpu": _cpu_model()},
         "e2e": {"value": round(val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
 
-# ----------------------------------------------------------------- our arm
-def workload_shape(g, mode, start, ms):
-    """Shape of the traversal the chain must follow: components,
-    the giant component's BFS levels from its RCM seed and its average front
-    (n_component / levels, C-14), Mnodes/s over the giant component only, and the
-    host.  Plain scipy/numpy on the host; not the oracle."""
-    import scipy.sparse as sp
-    from scipy.sparse.csgraph import breadth_first_order, connected_components
-    n = g.n
-    a = sp.csr_matrix((np.ones(g.nnz, dtype=np.int8), g.col_idx, g.row_ptr), shape=(n, n))
-    ncomp, lab = connected_components(a, directed=False)
-    sizes = np.bincount(lab)
-    giant = int(np.argmax(sizes))
-    deg = np.diff(g.row_ptr)
-    members = np.nonzero(lab == giant)[0]
-    if mode == 0 and lab[start] == giant:
-        seed = int(start)
-    else:   # MIN_DEGREE / C-6: min (valence, id) of the component
-        seed = int(members[np.lexsort((members, deg[members]))[0]])
-    order, pred = breadth_first_order(a, seed, directed=False, return_predecessors=True)
-    depth = np.zeros(n, dtype=np.int32)
-    for v in order[1:]:
-        depth[v] = depth[pred[v]] + 1
-    levels = int(depth[order].max()) + 1
-    cpu = ""
+# ----------------------------------------------------------------- helpers
+def hop_probe(rcm, nsm: int, iters: int = 400):
+    """SURVEY §8(d) chain-latency bound: one-way block-to-block hand-off from SM
+    0 to every other SM; the two dies show up as two latency clusters."""
     try:
-        cpu = next(l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name"))
-    except Exception:
-        pass
-    return {"components": int(ncomp), "giant_component_nodes": int(sizes[giant]), "levels_giant": levels,
-            "avg_front_giant": round(int(sizes[giant]) / levels, 1),
-            "giant_mnodes_per_s": round(int(sizes[giant]) / (ms * 1e-3) / 1e6, 3),
-            "us_per_level_giant": round(1e3 * ms / levels, 2),
-            "host_cpu": cpu, "host_cores": os.cpu_count()}
+        t = np.array([rcm.rcm_probe_hop(0, j, iters) for j in range(1, nsm)])
+        t = t[t > 0]
+        if t.size < 4:
+            return {"unavailable": "probe could not place blocks"}
+        thr = (t.min() + t.max()) / 2
+        near, far = t[t <= thr], t[t > thr]
+        return {"t_hop_ns_same_die": round(float(np.median(near)), 1),
+                "t_hop_ns_cross_die": round(float(np.median(far)), 1) if far.size else None,
+                "sm_pairs": int(t.size), "cross_die_pairs": int(far.size),
+                "how": f"SM0 -> SMj ping-pong, {iters} round trips, st.release.gpu / relaxed poll + fence.acq_rel"}
+    except Exception as ex:
+        return {"unavailable": str(ex)[:120]}
 
 
-def cpu_batch_context(g, mode, start, ref, runs: int = 3):
-    """The paper's CPU-BATCH (NEXT-4, libcpubatch.so: Alg. 5 on std::thread) on
-    every host core, full workload, median of `runs`: context for the paper's
-    multicore numbers, not a baseline of the GPU kernel."""
-    try:
-        from paper_conf_ipps_mlakarwps21_b200 import cpu_batch
-        cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else os.cpu_count()
-        ts, ok = [], True
-        for _ in range(runs):
-            t0 = time.perf_counter()
-            perm = cpu_batch.rcm_cpu_batch(g.row_ptr, g.col_idx, mode, start, threads=cores)
-            ts.append(time.perf_counter() - t0)
-            ok = ok and bool(np.array_equal(perm, ref))
-        sec = statistics.median(ts)
-        return {"value": round(g.n / sec / 1e6, 3), "unit": "Mnodes/s", "cores": cores, "kind": "cpu_batch",
-                "ms": round(1e3 * sec, 3), "parity_vs_oracle": "bit-identical" if ok else "MISMATCH",
-                "sample": f"full workload graph, median of {runs} runs"}
-    except Exception as exc:   # context only: never fails the bench line
-        return {"unavailable": str(exc)[:200]}
-
-
-def run_ours(args, rank: int, world: int, local_rank: int):
+def time_events(fn, steps, stream, flush=None):
     import torch
-    import paper_conf_ipps_mlakarwps21_b200 as rcm
+    evs = []
+    for _ in range(steps):
+        if flush is not None:
+            flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fn()
+        e1.record(stream)
+        evs.append((e0, e1))
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) for a, b in evs]
 
-    dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
-    g, mode, start, name = load_workload(args.config)
+
+# ------------------------------------------------- single graphs (C1-C4)
+def single_graph(rcm, cfg: int, steps: int, warmup: int, dev, world: int = 1, dist=None, hop=None,
+                 full_line: bool = False):
+    """One connected-graph config through rcm_reorder: device time, e2e, parity,
+    roofline; on rank 0 also the oracle's time."""
+    import torch
+    import synth
+    g, mode, start = synth.config_graph(cfg)
     n, nnz = g.n, g.nnz
     rp_h = torch.from_numpy(g.row_ptr).pin_memory()
     ci_h = torch.from_numpy(g.col_idx).pin_memory()
-    rp = rp_h.to(dev)
-    ci = ci_h.to(dev)
+    rp, ci = rp_h.to(dev), ci_h.to(dev)
     perm = torch.empty(n, dtype=torch.int32, device=dev)
     plan = rcm.Plan(n, nnz, collect_stats=0, **_plan_env())
     stream = torch.cuda.current_stream()
@@ -259,78 +255,68 @@ def run_ours(args, rank: int, world: int, local_rank: int):
     def step():
         rcm.rcm_reorder(plan.handle, n, nnz, rp, ci, mode, start, perm)
 
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         step()
-    st = rcm.rcm_sync_status(plan.handle)
-    if st != 0:
-        raise RuntimeError(f"rcm_reorder failed: {rcm.STATUS.get(st)}")
-
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
+    if rcm.rcm_sync_status(plan.handle) != 0:
+        raise RuntimeError("rcm_reorder failed")
+    if dist is not None:
         dist.barrier()
     torch.cuda.synchronize()
-    sampler = ClockSampler(local_rank) if rank == 0 else None
-    if sampler:
-        sampler.start()
-    evs = []
-    for _ in range(args.steps):
-        flush.zero_()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        step()
-        e1.record(stream)
-        evs.append((e0, e1))
-    torch.cuda.synchronize()
-    step_ms = [a.elapsed_time(b) for a, b in evs]
-    dev_ms = sum(step_ms)
+    sampler = ClockSampler(dev.index or 0)
+    sampler.start()
+    ms_list = time_events(step, steps, stream, flush)
+    clocks = sampler.stop()
+    dev_ms = sum(ms_list)
     if dist is not None:
         t = torch.tensor([dev_ms], device=dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.barrier()
         dev_ms = float(t.item())
-    clocks = sampler.stop() if sampler else None
-    st = rcm.rcm_sync_status(plan.handle)
-    if st != 0:
-        raise RuntimeError(f"rcm_reorder failed: {rcm.STATUS.get(st)}")
+    if rcm.rcm_sync_status(plan.handle) != 0:
+        raise RuntimeError("rcm_reorder failed")
     phases = plan.timing()
-
-    # one stats run (counters off in the timed loop)
     splan = rcm.Plan(n, nnz, collect_stats=1)
     splan.reorder(rp, ci, mode, start)
     stats = splan.stats()
     info = splan.info()
     splan.close()
-
-    # e2e through the public API: pinned host CSR in, permutation out, per step
+    # e2e: pinned host CSR in, permutation out, every step
     perm_h = torch.empty(n, dtype=torch.int32).pin_memory()
-    e2e_evs = []
-    if dist is not None:
-        dist.barrier()
-    torch.cuda.synchronize()
-    for _ in range(args.steps):
-        flush.zero_()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
+
+    def e2e_step():
         rp.copy_(rp_h, non_blocking=True)
         ci.copy_(ci_h, non_blocking=True)
         step()
         perm_h.copy_(perm, non_blocking=True)
-        e1.record(stream)
-        e2e_evs.append((e0, e1))
-    torch.cuda.synchronize()
-    e2e_ms = sum(a.elapsed_time(b) for a, b in e2e_evs)
-    if dist is not None:
-        t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_ms = float(t.item())
-
-    if rank != 0:
-        plan.close()
-        return
-    # parity of the benchmarked output against the oracle (and the CPU baseline)
+    e2e_ms = sum(time_events(e2e_step, steps, stream, flush)) / steps
+    # start finder (timed apart, as Table I does)
+    gl_out = torch.empty(1, dtype=torch.int32, device=dev)
+    s0 = int(np.argmax(np.diff(g.row_ptr)))
+    gl_ms = statistics.median(time_events(
+        lambda: rcm.rcm_find_pseudo_peripheral(plan.handle, n, nnz, rp, ci, s0, gl_out), 3, stream))
+    gl_node = int(gl_out.item())
+    plan.close()
+    ms = dev_ms / steps
+    res = {"workload": CONFIG_NAMES[cfg], "n": n, "nnz": nnz, "ms": round(ms, 4),
+           "mnodes_per_s": round(n / (ms * 1e-3) / 1e6, 3),
+           "e2e_mnodes_per_s": round(n / (e2e_ms * 1e-3) / 1e6, 3), "e2e_ms": round(e2e_ms, 4),
+           "phases_ms": {k: round(v, 4) for k, v in phases.items()}, "stats": stats, "plan": info,
+           "start_finder_ms": round(gl_ms, 4), "start_finder_from": s0, "start_finder_node": gl_node,
+           "clocks": clocks}
+    peak, _ = _peaks()
+    csr_once = 4 * (n + 1) + 4 * nnz
+    alg = csr_once + 28 * n
+    kern_ms = statistics.mean(ms_list)
+    res["roofline"] = {"bound": "hbm", "achieved": round(alg / (kern_ms * 1e-3) / 1e9, 3), "peak": peak,
+                       "unit": "GB/s", "frac": round(alg / (kern_ms * 1e-3) / 1e9 / peak, 6),
+                       "traffic": traffic_from_profile(f"c{cfg}"), "kernel": "k_main",
+                       "algorithmic_bytes": alg, "csr_once_bytes": csr_once,
+                       "csr_once_frac": round(csr_once / (kern_ms * 1e-3) / 1e9 / peak, 6)}
+    executed = max(1, stats.get("batches_executed", 1))
+    res["chain"] = {"batches_executed": stats.get("batches_executed"),
+                    "us_per_executed_batch": round(1e3 * phases["traversal_ms"] / executed, 3)}
+    if hop and "t_hop_ns_same_die" in hop:
+        res["chain"]["t_hop_us_same_die"] = round(hop["t_hop_ns_same_die"] / 1e3, 3)
+    # parity of the benchmarked output against the oracle
     import oracle
     oracle.build()
     ots = []
@@ -340,108 +326,61 @@ def run_ours(args, rank: int, world: int, local_rank: int):
         ref = oracle.rcm(g.row_ptr, g.col_idx, mode, start)
         ots.append(time.perf_counter() - t0)
     o_ms = 1e3 * statistics.median(ots)
-    got = perm_h.numpy()
-    parity = bool(np.array_equal(got, ref))
-
-    ms = dev_ms / args.steps
-    value = world * n / (ms * 1e-3) / 1e6
-    e2e_val = world * n / (e2e_ms / args.steps * 1e-3) / 1e6
-    peak, peak_kind = _peaks()
-    csr_once = 4 * (n + 1) + 4 * nnz
-    alg_bytes = csr_once + 28 * n
-    kern_ms = statistics.mean(step_ms)           # the step is exactly one k_main launch
-    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
-    executed = max(1, stats["batches_executed"])
-    line = {
-        "metric": "RCM Mnodes/s (ms/matrix in config) vs host serial RCM; % of HBM roofline",
-        "value": round(value, 3), "unit": "Mnodes/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "i32", "data": "synthetic",
-        "config": {"workload": name, "n": n, "nnz": nnz, "ms_per_matrix": round(ms, 4),
-                   "l2": "flushed before every timed step (256 MB write)",
-                   "parallelism": "replicas only" if world > 1 else "single GPU",
-                   "parity_vs_oracle": "bit-identical" if parity else "MISMATCH",
-                   "plan": info},
-        "roofline": {"bound": "hbm", "achieved": round(achieved, 3), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 6), "traffic": traffic_from_profile(args.config),
-                     "peak_kind": peak_kind, "kernel": "k_main",
-                     "algorithmic_bytes": alg_bytes,
-                     "csr_once_bytes": csr_once,
-                     "csr_once_frac": round(csr_once / (kern_ms * 1e-3) / 1e9 / peak, 6)},
-        "cpu_baseline": {"value": round(n / (o_ms * 1e-3) / 1e6, 3), "unit": "Mnodes/s", "cores": 1,
-                         "kind": "oracle", "ms": round(o_ms, 3),
-                         "sample": "full workload graph, serial oracle, median of 3 runs"},
-        "speedup_vs_oracle": round(o_ms / ms, 2),
-        "cpu_batch": cpu_batch_context(g, mode, start, ref) if rank == 0 else None,
-        "workload_shape": workload_shape(g, mode, start, ms) if rank == 0 else None,
-        "e2e": {"value": round(e2e_val, 3), "unit": "Mnodes/s", "h2d_bytes_per_step": 4 * (n + 1) + 4 * nnz,
-                "d2h_bytes_per_step": 4 * n, "ms_per_step": round(e2e_ms / args.steps, 4)},
-        "gpu_launches": args.steps,
-        "clocks": clocks,
-        "phases_ms": {k: round(v, 4) for k, v in phases.items()},
-        "stats": stats,
-        "chain": {"ms_per_executed_batch": round(phases["traversal_ms"] / executed, 5)},
-    }
-    print(json.dumps(line), flush=True)
-    plan.close()
+    res["parity_vs_oracle"] = "bit-identical" if np.array_equal(perm_h.numpy(), ref) else "MISMATCH"
+    res["start_finder_parity"] = ("identical to oracle.gl" if gl_node == oracle.gl(g.row_ptr, g.col_idx, s0)
+                                  else "MISMATCH")
+    res["oracle_ms"] = round(o_ms, 3)
+    res["oracle_mnodes_per_s"] = round(n / (o_ms * 1e-3) / 1e6, 3)
+    res["speedup_vs_oracle"] = round(o_ms / ms, 2)
+    return res
 
 
 # ---------------------------------------------------- config 5 (batched)
-def c5_sample(num, count, seed=12345):
-    """Matrices sampled for host-side parity / CPU baseline (largest, smallest, random)."""
-    import synth
-    sizes = synth.c5_sizes(num)
-    rng = np.random.default_rng(seed)
-    pick = {int(np.argmax(sizes)), int(np.argmin(sizes))}
-    pick.update(int(k) for k in rng.choice(num, count, replace=False))
-    return sorted(pick)
-
-
-def run_ours_c5(args, rank: int, world: int, local_rank: int):
+def run_c5(args, rank: int, world: int, local_rank: int, dist):
     import torch
     import synth
     import synth.device as sd
     import paper_conf_ipps_mlakarwps21_b200 as rcm
+    from paper_conf_ipps_mlakarwps21_b200 import shard
 
     dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
     num = args.num_mats
     sizes = synth.c5_sizes(num)
     _, n_all, nnz_all = sd.c5_specs(np.arange(num), sizes)
-    from paper_conf_ipps_mlakarwps21_b200 import shard
     parts = shard.lpt_partition(nnz_all, world)           # deterministic LPT on nnz
     mine = parts[rank]
     b = sd.c5_generate(mine, num=num, device=dev)
     total, total_nnz = b["total"], b["total_nnz"]
-    plan = rcm.Plan(total, total_nnz, **_plan_env())
+    opts = dict(flags=rcm.RCM_FLAG_BATCHED_ONLY)
+    opts.update(_plan_env())
+    plan = rcm.Plan(total, total_nnz, **opts)
     perm = torch.empty(total, dtype=torch.int32, device=dev)
     stream = torch.cuda.current_stream()
     part_tot = [int(n_all[p].sum()) for p in parts]
-
-    def gather():
-        # NCCL gather of the per-rank permutations into rank 0 (grouped send/recv)
-        return shard.gather_to_root(perm, part_tot, rank, world)
 
     def step():
         rcm.rcm_reorder_batched(plan.handle, len(mine), total, total_nnz, b["node_off"], b["nnz_off"],
                                 b["row_ptr_local"], b["col_idx_local"], rcm.RCM_START_MIN_DEGREE, None, perm)
 
+    gathered = None
+
+    def gather():
+        nonlocal gathered
+        gathered = shard.gather_to_root(perm, part_tot, rank, world)   # NCCL grouped send/recv
+
     for _ in range(args.warmup):
         step()
         if world > 1:
             gather()
-    st = rcm.rcm_sync_status(plan.handle)
-    if st != 0:
-        raise RuntimeError(f"rcm_reorder_batched failed: {rcm.STATUS.get(st)}")
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
+    if rcm.rcm_sync_status(plan.handle) != 0:
+        raise RuntimeError("rcm_reorder_batched failed")
+    if dist is not None:
         dist.barrier()
     torch.cuda.synchronize()
     sampler = ClockSampler(local_rank) if rank == 0 else None
     if sampler:
         sampler.start()
-    evs, gevs = [], []
+    evs = []
     for _ in range(args.steps):
         e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
         e0.record(stream)
@@ -452,6 +391,7 @@ def run_ours_c5(args, rank: int, world: int, local_rank: int):
         e2.record(stream)
         evs.append((e0, e1, e2))
     torch.cuda.synchronize()
+    clocks = sampler.stop() if sampler else None
     step_ms = [a.elapsed_time(c) for a, _, c in evs]
     kern_ms = [a.elapsed_time(bb) for a, bb, _ in evs]
     gath_ms = [bb.elapsed_time(c) for _, bb, c in evs]
@@ -459,14 +399,25 @@ def run_ours_c5(args, rank: int, world: int, local_rank: int):
     if dist is not None:
         t = torch.tensor([dev_ms], device=dev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.barrier()
         dev_ms = float(t.item())
-    clocks = sampler.stop() if sampler else None
-    st = rcm.rcm_sync_status(plan.handle)
-    if st != 0:
-        raise RuntimeError(f"rcm_reorder_batched failed: {rcm.STATUS.get(st)}")
+    if rcm.rcm_sync_status(plan.handle) != 0:
+        raise RuntimeError("rcm_reorder_batched failed")
     phases = plan.timing()
-    # e2e through the public API: the batch CSR from pinned host memory, the
+    plan_info = plan.info()
+    # one counters run (off in the timed loop)
+    splan = rcm.Plan(total, total_nnz, collect_stats=1, **opts)
+    sperm = torch.empty_like(perm)
+    splan.reorder_batched(b["node_off"], b["nnz_off"], b["row_ptr_local"], b["col_idx_local"], total, total_nnz,
+                          perm_local=sperm)
+    stats = splan.stats()
+    # start finder: the same batch with the GL finder per matrix, timed apart
+    pp_ms = statistics.median(time_events(
+        lambda: rcm.rcm_reorder_batched(splan.handle, len(mine), total, total_nnz, b["node_off"], b["nnz_off"],
+                                        b["row_ptr_local"], b["col_idx_local"],
+                                        rcm.RCM_START_PSEUDO_PERIPHERAL, None, sperm), 3, stream))
+    splan.close()
+    del sperm
+    # e2e through the public API: batch CSR from pinned host memory, the
     # permutations back to pinned host memory, every step
     e2e = None
     try:
@@ -479,19 +430,15 @@ def run_ours_c5(args, rank: int, world: int, local_rank: int):
         if dist is not None:
             dist.barrier()
         torch.cuda.synchronize()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(e2e_steps):
+
+        def e2e_step():
             b["row_ptr_local"].copy_(rp_h, non_blocking=True)
             b["col_idx_local"].copy_(ci_h, non_blocking=True)
             step()
             perm_h.copy_(perm, non_blocking=True)
             if world > 1:
                 gather()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        e2e_ms = e0.elapsed_time(e1) / e2e_steps
+        e2e_ms = sum(time_events(e2e_step, e2e_steps, stream)) / e2e_steps
         if dist is not None:
             t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -499,93 +446,165 @@ def run_ours_c5(args, rank: int, world: int, local_rank: int):
         e2e = {"value": round(int(n_all.sum()) / (e2e_ms * 1e-3) / 1e6, 3), "unit": "Mnodes/s",
                "h2d_bytes_per_step": 4 * (rp_h.numel() + ci_h.numel()), "d2h_bytes_per_step": 4 * total,
                "ms_per_step": round(e2e_ms, 4), "steps": e2e_steps}
-        del rp_h, ci_h
+        del rp_h, ci_h, perm_h
     except RuntimeError as ex:   # pinned host memory for ~11 GB may be unavailable
         e2e = {"value": None, "unit": "Mnodes/s", "unavailable": str(ex)[:120]}
+    if world > 1:
+        gather()   # the permutations of the last step, for the parity check
+    torch.cuda.synchronize()
+    plan.close()
     if rank != 0:
-        plan.close()
-        return
-    # parity on sampled matrices of this rank's share (host oracle on numpy twins)
+        return None
+    # parity: EVERY matrix of EVERY rank (assembled from the NCCL gather) against
+    # the serial oracle on all host cores -- also the cpu_baseline
     import oracle
     oracle.build()
-    perm_h = perm.cpu().numpy()
-    pos_of = {int(k): i for i, k in enumerate(mine)}
-    sample = [k for k in c5_sample(num, 24) if k in pos_of][:16]
-    parity_ok, o_nodes, o_sec = True, 0, 0.0
-    for k in sample:
-        i = pos_of[k]
-        g = synth.c5_matrix(k, int(sizes[k]))
+    got = shard.assemble([x.cpu().numpy() for x in gathered] if world > 1 else [perm.cpu().numpy()], parts, n_all)
+    del b
+    torch.cuda.empty_cache()
+    cores = _cores()
+    bad, o_sec, o_nodes = 0, 0.0, 0
+    for r in range(world):
+        br = sd.c5_generate(parts[r], num=num, device=dev)
+        rp = br["row_ptr_local"].cpu().numpy()
+        ci = br["col_idx_local"].cpu().numpy()
+        no, zo = br["node_off_h"], br["nnz_off_h"]
+        del br
+        torch.cuda.empty_cache()
         t0 = time.perf_counter()
-        ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE)
+        ref = oracle.rcm_batched(no, zo, rp, ci, oracle.MIN_DEGREE, threads=cores)
         o_sec += time.perf_counter() - t0
-        o_nodes += g.n
-        a, e = int(b["node_off_h"][i]), int(b["node_off_h"][i + 1])
-        parity_ok &= bool(np.array_equal(perm_h[a:e], ref))
+        o_nodes += int(no[-1])
+        for i, k in enumerate(parts[r]):
+            bad += not np.array_equal(got[k], ref[no[i]:no[i + 1]])
+        del rp, ci, ref
     ms = dev_ms / args.steps
     nodes_all = int(n_all.sum())
     value = nodes_all / (ms * 1e-3) / 1e6
     peak, peak_kind = _peaks()
-    nnz_mine = total_nnz
-    csr_once = 4 * (total + len(mine)) + 4 * nnz_mine
+    csr_once = 4 * (total + len(mine)) + 4 * total_nnz
     alg_bytes = csr_once + 28 * total
     km = statistics.mean(kern_ms)
     achieved = alg_bytes / (km * 1e-3) / 1e9
+    executed = max(1, stats.get("batches_executed", 1))
     line = {
-        "metric": "RCM Mnodes/s (ms/matrix in config) vs host serial RCM; % of HBM roofline",
+        "metric": _metric(),
         "value": round(value, 3), "unit": "Mnodes/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms, 4), "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": None, "dtype": "i32", "data": "synthetic",
-        "config": {"workload": f"C5 batch of {num} 2D/3D mesh matrices (1k-100k nodes), MIN_DEGREE per matrix",
-                   "matrices": num, "nodes": nodes_all, "nnz": int(nnz_all.sum()),
-                   "ms_per_matrix": round(ms / num, 6), "l2": "inputs (11 GB) larger than L2",
-                   "parallelism": f"matrices sharded over {world} GPU(s), LPT on nnz; NCCL gather to rank 0",
-                   "parity_vs_oracle": ("bit-identical" if parity_ok else "MISMATCH") +
-                                       f" on {len(sample)} sampled matrices of rank 0"},
+        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "i32",
+        "data": "synthetic (seeded, generated on the device)",
+        "config": {"workload": CONFIG_NAMES[5], "matrices": num, "nodes": nodes_all, "nnz": int(nnz_all.sum()),
+                   "ms_per_matrix": round(ms / num, 6),
+                   "l2": "not flushed: inputs (11 GB) are larger than the 126 MB L2",
+                   "parallelism": (f"matrices sharded over {world} GPUs (LPT on nnz), NCCL gather of the "
+                                   "permutations into rank 0 inside the step") if world > 1 else "single GPU",
+                   "parity_vs_oracle": (f"bit-identical on all {num} matrices" if bad == 0
+                                        else f"MISMATCH on {bad} of {num} matrices"),
+                   "plan": plan_info},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 3), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 6), "traffic": None, "peak_kind": peak_kind,
-                     "kernel": "k_main (batched)", "algorithmic_bytes": alg_bytes, "csr_once_bytes": csr_once},
-        "cpu_baseline": {"value": round(o_nodes / o_sec / 1e6, 3), "unit": "Mnodes/s", "cores": 1,
-                         "kind": "oracle", "sample": f"{len(sample)} matrices ({o_nodes} nodes), serial oracle"},
+                     "frac": round(achieved / peak, 6), "traffic": traffic_from_profile("c5"),
+                     "peak_kind": peak_kind, "kernel": "k_solo (+ k_solo_order, 1 block)",
+                     "algorithmic_bytes": alg_bytes, "csr_once_bytes": csr_once,
+                     "csr_once_frac": round(csr_once / (km * 1e-3) / 1e9 / peak, 6)},
+        "cpu_baseline": {"value": round(o_nodes / o_sec / 1e6, 3), "unit": "Mnodes/s", "cores": cores,
+                         "kind": "oracle", "ms": round(1e3 * o_sec, 1),
+                         "sample": f"all {num} matrices ({o_nodes} nodes), serial oracle per matrix on a "
+                                   f"{cores}-thread pool (the parity run)", "host_cpu": _cpu_model()},
+        "speedup_vs_oracle": round((1e3 * o_sec) / ms, 2),
         "e2e": e2e,
-        "gpu_launches": args.steps,
-        "gather_ms": round(statistics.mean(gath_ms), 4),
+        "gpu_launches": 2 * args.steps,
+        "gather_ms": round(statistics.mean(gath_ms), 4) if world > 1 else 0.0,
         "kernel_ms": round(km, 4),
         "clocks": clocks,
         "phases_ms": {k: round(v, 4) for k, v in phases.items()},
+        "stats": stats,
+        "batch": {"executed": stats.get("batches_executed"),
+                  "us_per_batch_per_block": round(1e3 * km * plan_info["solo_blocks"] / executed, 3),
+                  "note": "k_solo time x resident blocks / batches: the per-batch latency of one block"},
+        "start_finder": {"pseudo_peripheral_step_ms": round(pp_ms, 4), "min_degree_step_ms": round(km, 4),
+                         "gl_ms": round(pp_ms - km, 4),
+                         "note": "same batch with RCM_START_PSEUDO_PERIPHERAL (GL per matrix) minus MIN_DEGREE"},
     }
-    print(json.dumps(line), flush=True)
-    plan.close()
+    return line
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--config", type=int, default=5)
     ap.add_argument("--num-mats", type=int, default=8192)
+    ap.add_argument("--no-secondary", action="store_true", help="skip the C4 / C2 lines (N = 1)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # self-launch N ranks (one process per GPU) on this node
+        import socket
+        with socket.socket() as s:
+            s.bind(("127.0.0.1", 0))
+            port = s.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+        os.execv(sys.executable, cmd)
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local_rank = int(os.environ.get("LOCAL_RANK", 0))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     if args.impl == "reference":
         run_reference(args, rank)
         return
+    import torch
+    torch.cuda.set_device(local_rank)
+    dist = None
     if world > 1:
-        import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
-    try:
-        if args.config == 5:
-            run_ours_c5(args, rank, world, local_rank)
-        else:
-            run_ours(args, rank, world, local_rank)
-    finally:
-        if world > 1:
-            import torch.distributed as dist
-            dist.destroy_process_group()
+    import paper_conf_ipps_mlakarwps21_b200 as rcm
+    dev = torch.device("cuda", local_rank)
+    hop = hop_probe(rcm, torch.cuda.get_device_properties(dev).multi_processor_count) if rank == 0 else None
+    if args.config == 5:
+        line = run_c5(args, rank, world, local_rank, dist)
+        if line is not None:
+            line["chain_latency"] = hop
+            if world == 1 and not args.no_secondary:
+                line["secondary"] = {f"C{c}": single_graph(rcm, c, 5, 2, dev, hop=hop) for c in (4, 2)}
+    else:
+        res = single_graph(rcm, args.config, args.steps, args.warmup, dev, world, dist, hop)
+        line = None
+        if rank == 0:
+            line = {"metric": _metric(), "value": res["mnodes_per_s"], "unit": "Mnodes/s", "n_gpus": world,
+                    "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms"],
+                    "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "i32",
+                    "data": "synthetic (seeded)",
+                    "config": {"workload": res["workload"], "n": res["n"], "nnz": res["nnz"],
+                               "ms_per_matrix": res["ms"], "l2": "flushed before every timed step (256 MB write)",
+                               "parallelism": ("replicas only: a connected graph stays on one GPU; value = n / "
+                                               "max-over-ranks time, not a scaling measurement")
+                               if world > 1 else "single GPU",
+                               "parity_vs_oracle": res["parity_vs_oracle"], "plan": res["plan"]},
+                    "roofline": res["roofline"],
+                    "cpu_baseline": {"value": res["oracle_mnodes_per_s"], "unit": "Mnodes/s", "cores": 1,
+                                     "kind": "oracle", "ms": res["oracle_ms"],
+                                     "sample": "full workload graph, serial oracle, median of 3 runs"},
+                    "speedup_vs_oracle": res["speedup_vs_oracle"],
+                    "e2e": {"value": res["e2e_mnodes_per_s"], "unit": "Mnodes/s",
+                            "h2d_bytes_per_step": 4 * (res["n"] + 1) + 4 * res["nnz"],
+                            "d2h_bytes_per_step": 4 * res["n"], "ms_per_step": res["e2e_ms"]},
+                    "gpu_launches": args.steps, "clocks": res["clocks"], "phases_ms": res["phases_ms"],
+                    "stats": res["stats"],
+                    "chain": res["chain"], "chain_latency": hop,
+                    "start_finder_ms": res["start_finder_ms"], "start_finder_parity": res["start_finder_parity"]}
+    if dist is not None:
+        dist.barrier()
+    if rank == 0 and line is not None:
+        print(json.dumps(line), flush=True)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
 
 
 if __name__ == "__main__":

@@ -26,6 +26,8 @@ RCM_FLAG_NO_SORT = 0x4
 RCM_FLAG_FORCE_CHAIN = 0x8
 RCM_FLAG_SERIAL_CHAIN = 0x10
 RCM_FLAG_LEVELED = 0x20
+RCM_FLAG_MULTI_BATCH = 0x40
+RCM_FLAG_BATCHED_ONLY = 0x80
 
 STATUS = {
     0: "RCM_OK", 1: "RCM_ERR_INVALID_ARGUMENT", 2: "RCM_ERR_BAD_CSR", 3: "RCM_ERR_NOT_SYMMETRIC",
@@ -36,7 +38,7 @@ STATUS = {
 # every symbol include/rcm.h declares
 EXPORTS = ["rcm_default_options", "rcm_plan_create", "rcm_reorder", "rcm_reorder_batched",
            "rcm_find_pseudo_peripheral", "rcm_sync_status", "rcm_get_stats", "rcm_get_timing", "rcm_plan_info",
-           "rcm_plan_destroy", "rcm_status_string"]
+           "rcm_plan_destroy", "rcm_status_string", "rcm_probe_hop"]
 
 
 class rcm_options_t(ctypes.Structure):
@@ -95,6 +97,8 @@ def _load():
     lib.rcm_get_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_double)]
     lib.rcm_plan_destroy.argtypes = [vp]
     lib.rcm_plan_destroy.restype = None
+    lib.rcm_probe_hop.argtypes = [i32, i32, i32, ctypes.POINTER(ctypes.c_double)]
+    lib.rcm_probe_hop.restype = i32
     lib.rcm_status_string.argtypes = [i32]
     lib.rcm_status_string.restype = ctypes.c_char_p
     for f in ("rcm_plan_create", "rcm_reorder", "rcm_reorder_batched", "rcm_find_pseudo_peripheral",
@@ -200,15 +204,22 @@ def rcm_get_timing(plan) -> dict:
 
 
 def rcm_plan_info(plan) -> dict:
-    a = (ctypes.c_int64 * 6)()
+    a = (ctypes.c_int64 * 8)()
     _check(_load().rcm_plan_info(plan, a), "rcm_plan_info")
-    return dict(zip(("blocks", "threads", "batch_nodes", "temp_elems", "smem_bytes", "queue_slots"),
-                    [int(x) for x in a]))
+    return dict(zip(("blocks", "threads", "batch_nodes", "temp_elems", "smem_bytes", "queue_slots",
+                     "solo_blocks", "solo_smem_bytes"), [int(x) for x in a]))
 
 
 def rcm_plan_destroy(plan) -> None:
     if plan:
         _load().rcm_plan_destroy(plan)
+
+
+def rcm_probe_hop(sm_a: int, sm_b: int, iters: int = 2000) -> float:
+    """One-way block-to-block hand-off time (ns) between SMs sm_a and sm_b."""
+    out = ctypes.c_double()
+    _check(_load().rcm_probe_hop(int(sm_a), int(sm_b), int(iters), ctypes.byref(out)), "rcm_probe_hop")
+    return float(out.value)
 
 
 def rcm_status_string(st: int) -> str:

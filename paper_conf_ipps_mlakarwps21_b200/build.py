@@ -8,9 +8,9 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librcm.so")
-SOURCES = ["rcm.cu", "k_main_inst.cu"]
+SOURCES = ["rcm.cu", "k_main_inst.cu", "k_solo.cu", "k_probe.cu"]
 HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh",
-           "rcm_leveled.cuh", "rcm_main.cuh"]
+           "rcm_leveled.cuh", "rcm_main.cuh", "rcm_solo.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-O2",
@@ -48,7 +48,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
     extra = _extra_defines()
     if verbose:
         extra = ["-Xptxas=-v", *extra]
-    jobs = [(os.path.join(BUILD_DIR, "rcm.o"), [os.path.join(CSRC, "rcm.cu")])]
+    jobs = [(os.path.join(BUILD_DIR, "rcm.o"), [os.path.join(CSRC, "rcm.cu")]),
+            (os.path.join(BUILD_DIR, "k_solo.o"), [os.path.join(CSRC, "k_solo.cu")]),
+            (os.path.join(BUILD_DIR, "k_probe.o"), [os.path.join(CSRC, "k_probe.cu")])]
     for bps, mb in KMAIN_VARIANTS:
         jobs.append((os.path.join(BUILD_DIR, f"k_main_{bps}_{mb}.o"),
                      [f"-DRCM_KBPS={bps}", f"-DRCM_KMB={mb}", os.path.join(CSRC, "k_main_inst.cu")]))
@@ -64,7 +66,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     for obj, _ in procs:
         os.replace(obj + f".tmp{os.getpid()}", obj)
     tmp = LIB + f".tmp{os.getpid()}"
-    subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-o", tmp,
+    subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-Xlinker", "--no-undefined", "-o", tmp,
                            *[obj for obj, _ in jobs]])
     os.replace(tmp, LIB)
     return LIB

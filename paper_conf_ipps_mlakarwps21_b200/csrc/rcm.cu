@@ -10,6 +10,7 @@
 
 #include "../../include/rcm.h"
 #include "rcm_components.cuh"
+#include "rcm_solo.cuh"
 
 using namespace rcm;
 
@@ -35,6 +36,14 @@ struct rcm_plan {
   int32_t trace_cap = 0;
   const void* kernel = nullptr;
   CompWS w{};
+  // batched / small-graph path (rcm_solo.cuh)
+  int solo_blocks = 0;
+  size_t solo_smem = 0;
+  int64_t mats_cap = 0, gvis_words = 0;
+  int32_t* order = nullptr;
+  uint32_t* gvis = nullptr;
+  int solo_BS = 256;
+  bool batched_only = false;
 };
 
 static rcm_status_t cuda_fail(cudaError_t e) {
@@ -67,7 +76,7 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
                   p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
@@ -87,10 +96,62 @@ extern "C" const void* rcm_kmain_ptr_1_0();
 extern "C" const void* rcm_kmain_ptr_2_0();
 extern "C" const void* rcm_kmain_ptr_1_1();
 extern "C" const void* rcm_kmain_ptr_2_1();
+extern "C" const void* rcm_ksolo_order_ptr();
+extern "C" const void* rcm_ksolo_ptr();
+extern "C" size_t rcm_ksolo_smem();
+extern "C" int rcm_ksolo_threads();
+extern "C" int rcm_ksolo_nmax();
 static const void* pick_kernel(int bps, bool mb) {
   static_assert(1024 / kThreads >= 2, "two 512-thread blocks per SM");
   if (mb) return bps >= 2 ? rcm_kmain_ptr_2_1() : rcm_kmain_ptr_1_1();
   return bps == 2 ? rcm_kmain_ptr_2_0() : rcm_kmain_ptr_1_0();
+}
+
+static rcm_status_t plan_alloc(rcm_plan* p) {
+  const rcm_options_t& o = p->opt;
+  const int64_t n = p->n_max;
+#define AL(ptr, bytes)                                          \
+  do {                                                          \
+    cudaError_t _e = cudaMalloc((void**)&(ptr), (size_t)(bytes)); \
+    if (_e != cudaSuccess) return cuda_fail(_e);                \
+  } while (0)
+  // shared by both paths
+  AL(p->ctl, sizeof(Ctl));
+  AL(p->stats, sizeof(Stats));
+  AL(p->dbg, 4 * 8 * 1024);
+  AL(p->spill, 8 * 2 * p->spill_cap);
+  // batched / small-graph path (rcm_solo.cuh)
+  AL(p->order, 4 * p->mats_cap);
+  AL(p->gvis, 4 * 2 * p->gvis_words);
+  if (!p->batched_only) {   // multi-block chain + components + GL finder
+    const int64_t tiles = (n + kSortTile - 1) / kSortTile + 1;
+    AL(p->word, 8 * n);
+    AL(p->o, 4 * n);
+    AL(p->desc, sizeof(Desc) * p->qcap);
+    AL(p->sig, sizeof(Sig) * (p->qcap + 1));
+    AL(p->chains, sizeof(Problem) * p->prob_cap);
+    AL(p->solos, sizeof(Problem) * p->prob_cap);
+    if (o.collect_stats == 3) {
+      p->trace_cap = (int32_t)std::min<int64_t>(p->qcap, 1 << 20);
+      AL(p->trace, 8 * kTraceW * (size_t)p->trace_cap);
+    }
+    AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
+    AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
+    AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kMaxBlocks));
+    AL(p->w.sctl, 4 * 64);
+    AL(p->w.lev, 4 * n); AL(p->w.front0, 4 * n); AL(p->w.front1, 4 * n);
+    AL(p->w.gctl, 4 * 64); AL(p->w.gkey, 8 * 64);
+    p->w.cap = n;
+    // descriptors / signals start with tag 0 (epochs start at 1)
+    CK(cudaMemset(p->desc, 0, sizeof(Desc) * p->qcap));
+    CK(cudaMemset(p->sig, 0, sizeof(Sig) * (p->qcap + 1)));
+  }
+#undef AL
+  CK(cudaMemset(p->ctl, 0, sizeof(Ctl)));
+  CK(cudaMemset(p->stats, 0, sizeof(Stats)));
+  CK(cudaMemset(p->dbg, 0, 4 * 8 * 1024));
+  CK(cudaDeviceSynchronize());
+  return RCM_OK;
 }
 
 extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t nnz_max,
@@ -100,104 +161,87 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   rcm_plan* p = new (std::nothrow) rcm_plan();
   if (!p) return RCM_ERR_OUT_OF_MEMORY;
   if (opt_in) p->opt = *opt_in;
-  rcm_options_t& o = p->opt;
-  if (o.batch_nodes < 0 || o.batch_nodes > kMaxBatchNodes || o.temp_elems < 0 || o.blocks_per_sm < 0 || o.blocks_per_sm > 4 ||
-      o.validate < 0 || o.validate > 2 || o.queue_capacity < 0) {
+  const rcm_options_t& o = p->opt;
+  if (o.batch_nodes < 0 || o.batch_nodes > kMaxBatchNodes || o.temp_elems < 0 || o.blocks_per_sm < 0 ||
+      o.blocks_per_sm > 4 || o.validate < 0 || o.validate > 2 || o.queue_capacity < 0) {
     delete p;
     return RCM_ERR_INVALID_ARGUMENT;
   }
   p->n_max = n_max;
   p->nnz_max = nnz_max;
+  p->batched_only = (o.flags & RCM_FLAG_BATCHED_ONLY) != 0;
   if (cudaGetDevice(&p->device) != cudaSuccess) { delete p; return RCM_ERR_CUDA; }
   cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->device);
   int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
-  const bool dense = !o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max;
-  // dense rows (FEM-like): smaller batches shorten the critical generation
-  // chain
-  p->BS = o.batch_nodes ? o.batch_nodes : dense ? 192 : 256;
-  const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
-  const size_t static_sh = 2 * sizeof(ShState) + 64;
-  const int nctx = (o.flags & RCM_FLAG_MULTI_BATCH) ? 2 : 1;   // batch contexts per block
-  // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per
-  // block), 10 B per slot (candidate key, local parent id)
-  const size_t per_block =
-      std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
-  int T = o.temp_elems;
-  if (!T) T = (int)((per_block / nctx - 16 - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
-  // dense: B_s rows of ~27 fit; the shared memory left over serves as L1
-  if (dense) T = std::min(T, 6144);
-  // sparse rows at the default occupancy: a budget past ~7.7 k candidates buys
-  // few extra parents per batch but takes the SM's L1 (r01d sweep, DESIGN.md §2.1
-  // "batch limits": C3 10.9 -> 9.6 ms, C5 94.7 -> ~70 ms, C4 unchanged)
-  else if (!o.temp_elems && !o.blocks_per_sm && nctx == 1) T = std::min(T, 7680);
-  if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
-    delete p;
-    return RCM_ERR_INVALID_ARGUMENT;
-  }
-  p->T = T;
-  p->smem = nctx == 1 ? smem_bytes(p->BS, T) : nctx * ((smem_bytes(p->BS, T) + 15) & ~size_t(15));
-  // one block per SM: the 128-register build (no spills); more: the 64-register build
-  p->kernel = pick_kernel(bps, nctx == 2);
-  if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
+  // ---- batched / small-graph path: many blocks per SM, shared-memory bitmap
+  p->solo_smem = rcm_ksolo_smem();
+  if (cudaFuncSetAttribute(rcm_ksolo_ptr(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->solo_smem) !=
+      cudaSuccess) {
     delete p;
     return RCM_ERR_CUDA;
   }
-  int occ = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, p->kernel, kThreads, p->smem);
-  if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
-  p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
-  if (p->nblocks > kMaxBlocks) p->nblocks = kMaxBlocks / p->num_sms * p->num_sms;   // beacon / scratch sizing
-  // queue bound: sum over generating batches of floor(N/B) + max(1, ceil(2V/T))
-  const int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
-  p->qcap = o.queue_capacity ? o.queue_capacity : std::min<int64_t>(qb, (1ll << 31) - 2);
-  p->prob_cap = std::max<int64_t>(1, n_max / 2 + 1);
+  int occ_s = 0;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, rcm_ksolo_ptr(), rcm_ksolo_threads(), p->solo_smem);
+  if (occ_s <= 0) { delete p; return RCM_ERR_CUDA; }
+  p->solo_blocks = occ_s * p->num_sms;
+  p->solo_BS = o.batch_nodes ? std::min(o.batch_nodes, rcm_ksolo_threads()) : rcm_ksolo_threads();
+  p->mats_cap = n_max + 1;
+  p->gvis_words = n_max / 32 + p->mats_cap + 2;
   p->spill_cap = n_max;
-  const int64_t n = n_max;
-  const int64_t tiles = (n + kSortTile - 1) / kSortTile + 1;
-  rcm_status_t st = RCM_OK;
-#define AL(ptr, bytes)                                        \
-  do {                                                        \
-    cudaError_t _e = cudaMalloc((void**)&(ptr), (bytes));     \
-    if (_e != cudaSuccess) { st = cuda_fail(_e); goto fail; } \
-  } while (0)
-  AL(p->word, 8 * n);
-  AL(p->o, 4 * n);
-  AL(p->desc, sizeof(Desc) * p->qcap);
-  AL(p->sig, sizeof(Sig) * (p->qcap + 1));
-  AL(p->ctl, sizeof(Ctl));
-  AL(p->stats, sizeof(Stats));
-  AL(p->chains, sizeof(Problem) * p->prob_cap);
-  AL(p->solos, sizeof(Problem) * p->prob_cap);
-  AL(p->pm_key, 8 * p->prob_cap);
-  AL(p->spill, 8 * 2 * p->spill_cap);
-  AL(p->dbg, 4 * 8 * 1024);
-  if (o.collect_stats == 3) {
-    p->trace_cap = (int32_t)std::min<int64_t>(p->qcap, 1 << 20);
-    AL(p->trace, 8 * kTraceW * (size_t)p->trace_cap);
+  // ---- multi-block chain path
+  if (!p->batched_only) {
+    const bool dense = !o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max;
+    // dense rows (FEM-like): smaller batches shorten the critical generation
+    // chain
+    p->BS = o.batch_nodes ? o.batch_nodes : dense ? 192 : 256;
+    const int bps = o.blocks_per_sm ? o.blocks_per_sm : 2;
+    const size_t static_sh = 2 * sizeof(ShState) + 64;
+    const int nctx = (o.flags & RCM_FLAG_MULTI_BATCH) ? 2 : 1;   // batch contexts per block
+    // T from the shared-memory budget of `bps` blocks per SM (1 KB reserved per
+    // block), 10 B per slot (candidate key, local parent id)
+    const size_t per_block =
+        std::min<size_t>((size_t)smem_sm / bps - 1024 - static_sh, (size_t)smem_optin - static_sh);
+    int T = o.temp_elems;
+    if (!T) T = (int)((per_block / nctx - 16 - smem_bytes(p->BS, 0)) / 10) / 256 * 256;
+    // dense: B_s rows of ~27 fit; the shared memory left over serves as L1
+    if (dense) T = std::min(T, 6144);
+    // sparse rows at the default occupancy: a budget past ~7.7 k candidates buys
+    // few extra parents per batch but takes the SM's L1 (r01d sweep, DESIGN.md
+    // "batch limits": C3 10.9 -> 9.6 ms, C4 unchanged)
+    else if (!o.temp_elems && !o.blocks_per_sm && nctx == 1) T = std::min(T, 7680);
+    if (T < 2304 || smem_bytes(p->BS, T) > (size_t)smem_optin - static_sh) {
+      delete p;
+      return RCM_ERR_INVALID_ARGUMENT;
+    }
+    p->T = T;
+    p->smem = nctx == 1 ? smem_bytes(p->BS, T) : nctx * ((smem_bytes(p->BS, T) + 15) & ~size_t(15));
+    // one block per SM: the 128-register build (no spills); more: the 64-register build
+    p->kernel = pick_kernel(bps, nctx == 2);
+    if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
+      delete p;
+      return RCM_ERR_CUDA;
+    }
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, p->kernel, kThreads, p->smem);
+    if (occ <= 0) { delete p; return RCM_ERR_CUDA; }
+    p->nblocks = std::min(occ, bps) * p->num_sms;   // persistent: every block co-resident
+    if (p->nblocks > kMaxBlocks) p->nblocks = kMaxBlocks / p->num_sms * p->num_sms;   // beacon / scratch sizing
+    // queue bound: sum over generating batches of floor(N/B) + max(1, ceil(2V/T))
+    const int64_t qb = 2 * n_max + n_max / p->BS + 2 * (nnz_max / T + 1) + 64;
+    // the Counted payload packs queue offsets in 30 bits (rcm_device.cuh sig_pack,
+    // rcm_lookback.cuh lb_pfx): the queue never exceeds 2^30 - 1 slots
+    p->qcap = std::min<int64_t>(o.queue_capacity ? o.queue_capacity : qb, (1ll << 30) - 1);
+    p->prob_cap = std::max<int64_t>(1, n_max / 2 + 1);
   }
-  AL(p->w.label, 4 * n); AL(p->w.ckey, 8 * n); AL(p->w.csize, 4 * n);
-  AL(p->w.keys0, 8 * n); AL(p->w.keys1, 8 * n); AL(p->w.vals0, 4 * n); AL(p->w.vals1, 4 * n);
-  AL(p->w.offs, 8 * (n + 1 + 1024)); AL(p->w.hist, 4 * std::max<int64_t>(256 * tiles, 4 * kMaxBlocks)); AL(p->w.sctl, 4 * 64);
-  AL(p->w.order, 4 * n); AL(p->w.lev, 4 * n); AL(p->w.front0, 4 * n); AL(p->w.front1, 4 * n);
-  AL(p->w.gctl, 4 * 64); AL(p->w.gkey, 8 * 64);
-#undef AL
-  p->w.cap = n;
-  // descriptors / signals start with tag 0 (epochs start at 1)
-  if (cudaMemset(p->desc, 0, sizeof(Desc) * p->qcap) != cudaSuccess ||
-      cudaMemset(p->sig, 0, sizeof(Sig) * (p->qcap + 1)) != cudaSuccess ||
-      cudaMemset(p->ctl, 0, sizeof(Ctl)) != cudaSuccess || cudaMemset(p->stats, 0, sizeof(Stats)) != cudaSuccess ||
-      cudaMemset(p->dbg, 0, 4 * 8 * 1024) != cudaSuccess ||
-      cudaDeviceSynchronize() != cudaSuccess) {
-    st = RCM_ERR_CUDA;
-    goto fail;
+  const rcm_status_t st = plan_alloc(p);
+  if (st != RCM_OK) {
+    rcm_plan_destroy(p);
+    return st;
   }
   *out = p;
   return RCM_OK;
-fail:
-  rcm_plan_destroy(p);
-  return st;
 }
 
 static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* col_idx, int32_t* perm,
@@ -258,6 +302,27 @@ static rcm_status_t launch_main(rcm_plan* p, const KParams& kp, const MainArgs& 
   return RCM_OK;
 }
 
+// The batched / small-graph path: k_solo_order (reset + largest-first order)
+// then k_solo on every SM (rcm_solo.cuh).  Regular launches: no block waits
+// for another, so co-residency is not required.
+static rcm_status_t launch_solo(rcm_plan* p, SoloArgs& sa, cudaStream_t s) {
+  sa.order = p->order;
+  sa.gvis = p->gvis;
+  sa.gvis_words = p->gvis_words;
+  sa.spill = p->spill;
+  sa.spill_cap = p->spill_cap;
+  sa.ctl = p->ctl;
+  sa.stats = p->stats;
+  sa.validate = p->opt.validate;
+  sa.collect_stats = p->opt.collect_stats;
+  sa.flags = p->opt.flags;
+  sa.BS = p->solo_BS;
+  void* args[] = {&sa};
+  CK(cudaLaunchKernel(rcm_ksolo_order_ptr(), dim3(1), dim3(1024), args, 0, s));
+  CK(cudaLaunchKernel(rcm_ksolo_ptr(), dim3(p->solo_blocks), dim3(rcm_ksolo_threads()), args, p->solo_smem, s));
+  return RCM_OK;
+}
+
 extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const int32_t* row_ptr,
                                     const int32_t* col_idx, rcm_start_t mode, int32_t start,
                                     int32_t* perm, int32_t* iperm, void* stream) {
@@ -265,6 +330,23 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   if (n > p->n_max || nnz > p->nnz_max || nnz >= (1ll << 31)) return RCM_ERR_INVALID_ARGUMENT;
   if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
   if (mode == RCM_START_FIXED && (start < 0 || start >= n)) return RCM_ERR_INVALID_ARGUMENT;
+  const int thr = p->opt.solo_threshold == 0 ? 4096 : p->opt.solo_threshold;
+  const bool solo = !(p->opt.flags & RCM_FLAG_FORCE_CHAIN) && thr > 0 && n <= thr;
+  if (solo) {   // one block orders the whole graph (small graphs, e.g. config 1)
+    SoloArgs sa;
+    std::memset(&sa, 0, sizeof(sa));
+    sa.row_ptr = row_ptr;
+    sa.col_idx = col_idx;
+    sa.perm = perm;
+    sa.iperm = iperm;
+    sa.num_mats = 1;
+    sa.n = n;
+    sa.nnz = nnz;
+    sa.mode = (int)mode;
+    sa.start = start;
+    return launch_solo(p, sa, (cudaStream_t)stream);
+  }
+  if (p->batched_only) return RCM_ERR_INVALID_ARGUMENT;   // no chain workspace in this plan
   KParams kp = make_kparams(p, row_ptr, col_idx, perm, iperm);
   if (!p->opt.batch_nodes && !p->opt.temp_elems && nnz >= 20ll * n) {
     // dense rows (FEM-like, average valence >= 20) on a plan sized for sparser
@@ -278,7 +360,6 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
   a.mode = (int)mode;
   a.start = start;
   a.vec = ((reinterpret_cast<uintptr_t>(row_ptr) & 15) == 0) ? 1 : 0;
-  a.solo = (!(p->opt.flags & RCM_FLAG_FORCE_CHAIN) && a.thr > 0 && n <= a.thr) ? 1 : 0;
   a.idbits = bits_for(n - 1 > 0 ? n - 1 : 1);
   return launch_main(p, kp, a, (cudaStream_t)stream);
 }
@@ -288,24 +369,24 @@ extern "C" rcm_status_t rcm_reorder_batched(rcm_plan_t p, int32_t num_mats, int6
                                             const int64_t* nnz_off, const int32_t* row_ptr_local,
                                             const int32_t* col_idx_local, rcm_start_t mode,
                                             const int32_t* starts, int32_t* perm_local, void* stream) {
-  if (!p || num_mats <= 0 || !node_off || !nnz_off || !row_ptr_local || !perm_local || total_nodes <= 0 ||
+  if (!p || num_mats <= 0 || !node_off || !nnz_off || !row_ptr_local || !perm_local || total_nodes < 0 ||
       total_nnz < 0 || (total_nnz > 0 && !col_idx_local))
     return RCM_ERR_INVALID_ARGUMENT;
-  if (total_nodes > p->n_max || total_nnz > p->nnz_max || num_mats > p->prob_cap) return RCM_ERR_INVALID_ARGUMENT;
+  if (total_nodes > p->n_max || total_nnz > p->nnz_max || num_mats > p->mats_cap - 1)
+    return RCM_ERR_INVALID_ARGUMENT;
   if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
   if (mode == RCM_START_FIXED && !starts) return RCM_ERR_INVALID_ARGUMENT;
-  KParams kp = make_kparams(p, row_ptr_local, col_idx_local, perm_local, nullptr);
-  MainArgs a = make_args(p);
-  a.batched = 1;
-  a.mode = (int)mode;
-  a.num_mats = num_mats;
-  a.total = total_nodes;
-  a.nnz = total_nnz;
-  a.node_off = node_off;
-  a.nnz_off = nnz_off;
-  a.starts = starts;
-  a.pm_key = p->pm_key;
-  return launch_main(p, kp, a, (cudaStream_t)stream);
+  SoloArgs sa;
+  std::memset(&sa, 0, sizeof(sa));
+  sa.row_ptr = row_ptr_local;
+  sa.col_idx = col_idx_local;
+  sa.perm = perm_local;
+  sa.node_off = node_off;
+  sa.nnz_off = nnz_off;
+  sa.starts = starts;
+  sa.num_mats = num_mats;
+  sa.mode = (int)mode;
+  return launch_solo(p, sa, (cudaStream_t)stream);
 }
 
 extern "C" rcm_status_t rcm_find_pseudo_peripheral(rcm_plan_t p, int32_t n, int64_t nnz,
@@ -313,7 +394,7 @@ extern "C" rcm_status_t rcm_find_pseudo_peripheral(rcm_plan_t p, int32_t n, int6
                                                    int32_t start, int32_t* out, void* stream) {
   if (!p || !row_ptr || !out || n <= 0 || start < 0 || start >= n || nnz < 0 || (nnz > 0 && !col_idx))
     return RCM_ERR_INVALID_ARGUMENT;
-  if (n > p->n_max || nnz > p->nnz_max) return RCM_ERR_INVALID_ARGUMENT;
+  if (n > p->n_max || nnz > p->nnz_max || p->batched_only) return RCM_ERR_INVALID_ARGUMENT;
   KParams kp = make_kparams(p, row_ptr, col_idx, nullptr, nullptr);
   MainArgs a = make_args(p);
   a.n = n;
@@ -408,7 +489,7 @@ extern "C" rcm_status_t rcm_debug_trace(rcm_plan_t p, int32_t cnt, unsigned long
 // Raw chain slot state (desc + both status words) for slots [lo, lo+cnt):
 // 6 int64 per slot.  Debug only; copied on a private stream.
 extern "C" rcm_status_t rcm_debug_slots(rcm_plan_t p, int32_t lo, int32_t cnt, long long* host_out) {
-  if (!p || !host_out || lo < 0 || cnt <= 0 || lo + cnt > p->qcap) return RCM_ERR_INVALID_ARGUMENT;
+  if (!p || !host_out || !p->sig || lo < 0 || cnt <= 0 || lo + cnt > p->qcap) return RCM_ERR_INVALID_ARGUMENT;
   cudaStream_t s;
   CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   Sig* sg = (Sig*)malloc(sizeof(Sig) * cnt);
@@ -433,13 +514,15 @@ extern "C" rcm_status_t rcm_debug_slots(rcm_plan_t p, int32_t lo, int32_t cnt, l
   return e == cudaSuccess ? RCM_OK : RCM_ERR_CUDA;
 }
 
-extern "C" rcm_status_t rcm_plan_info(rcm_plan_t p, int64_t* out6) {
-  if (!p || !out6) return RCM_ERR_INVALID_ARGUMENT;
-  out6[0] = p->nblocks;
-  out6[1] = kThreads;
-  out6[2] = p->BS;
-  out6[3] = p->T;
-  out6[4] = (int64_t)p->smem;
-  out6[5] = p->qcap;
+extern "C" rcm_status_t rcm_plan_info(rcm_plan_t p, int64_t* out8) {
+  if (!p || !out8) return RCM_ERR_INVALID_ARGUMENT;
+  out8[0] = p->nblocks;
+  out8[1] = kThreads;
+  out8[2] = p->BS;
+  out8[3] = p->T;
+  out8[4] = (int64_t)p->smem;
+  out8[5] = p->qcap;
+  out8[6] = p->solo_blocks;
+  out8[7] = (int64_t)p->solo_smem;
   return RCM_OK;
 }

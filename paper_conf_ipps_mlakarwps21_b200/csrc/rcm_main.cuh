@@ -85,40 +85,6 @@ static __device__ void validate_sym_phase(const KParams& kp, int n) {
   if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicCAS(&kp.ctl->status, 0, ST_NOT_SYM);
 }
 
-// Batched prologue: per matrix k, local valences and the per-matrix argmin.
-static __device__ void prologue_batched_phase(const KParams& kp, const MainArgs& a) {
-  const long long stride = (long long)gthreads(kp);
-  for (long long base = (long long)blockIdx.x * kThreads; base < a.total; base += stride) {
-    const long long g = base + threadIdx.x;   // warp-uniform loop; lanes past the end idle
-    const bool valid = g < a.total;
-    int k = -1;
-    unsigned long long key = kKeyMax;
-    if (valid) {
-      int lo = 0, hi = a.num_mats - 1;         // matrix of g: largest k with node_off[k] <= g
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (__ldg(a.node_off + mid) <= g) lo = mid; else hi = mid - 1;
-      }
-      k = lo;
-      const int v = (int)(g - __ldg(a.node_off + k));
-      const int d = max(__ldg(kp.row_ptr + g + k + 1) - __ldg(kp.row_ptr + g + k), 0);
-      kp.word[g] = ((unsigned long long)kInf << 32) | (uint32_t)d;
-      key = ((unsigned long long)(uint32_t)d << 32) | (uint32_t)v;
-    }
-    // lanes of one matrix are contiguous: a segmented shuffle-down min leaves
-    // the segment minimum in its first lane
-    const unsigned peers = __match_any_sync(0xffffffffu, k);
-    unsigned long long m = key;
-    const int lane = threadIdx.x & 31;
-    for (int off = 1; off < 32; off <<= 1) {
-      const unsigned long long o2 = __shfl_down_sync(0xffffffffu, m, off);
-      const int ko = __shfl_down_sync(0xffffffffu, k, off);
-      if (lane + off < 32 && ko == k && o2 < m) m = o2;
-    }
-    if (valid && lane == __ffs(peers) - 1) atomicMin(a.pm_key + k, m);
-  }
-}
-
 // The scheduling phase: every chain problem in turn on all blocks (grid
 // barrier between chains), then the solo problems, one per block at a time.
 template <bool kMB>
@@ -185,17 +151,12 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
     c->solo_next = 0; c->n_chain = 0; c->n_solo = 0; c->n_comp = 0; c->spill_cursor = 0; c->incomplete = 0;
     if (kp.collect_stats) *kp.stats = Stats{};
   }
-  if (a.batched)
-    for (int k = gtid(); k < a.num_mats; k += G) a.pm_key[k] = kKeyMax;
-  if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.gl_only) {
-    const long long nn = a.batched ? a.total : a.n;
-    for (long long v = gtid(); v < nn; v += G) a.w.lev[v] = -1;
-  }
+  if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.gl_only)
+    for (long long v = gtid(); v < a.n; v += G) a.w.lev[v] = -1;
   grid_barrier(kp);
   // ---- phase 1: prologue (a1)
-  if (a.batched) prologue_batched_phase(kp, a);
-  else prologue_phase(kp, a, sh);
-  if (!a.batched && a.validate == 2) validate_sym_phase(kp, a.n);
+  prologue_phase(kp, a, sh);
+  if (a.validate == 2) validate_sym_phase(kp, a.n);
   grid_barrier(kp);
   stamp(kp, 1);
   if (ld_cg_s32(&kp.ctl->status)) return;   // read after a barrier: uniform across blocks
@@ -206,46 +167,15 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
     return;
   }
   // ---- phase 2: problems
-  const int gl_flag = a.mode == RCM_START_PSEUDO_PERIPHERAL ? 2 : 0;
-  if (a.batched) {
-    // LPT: largest matrices first (solo workers dequeue in this order)
-    for (int k = gtid(); k < a.num_mats; k += G) {
-      const long long sz = a.node_off[k + 1] - a.node_off[k];
-      a.w.keys0[k] = ((unsigned long long)(0xffffffffu - (uint32_t)sz) << 32) | (uint32_t)k;
-      a.w.vals0[k] = k;
-    }
-    if (gtid() == 0) { a.w.sctl[0] = a.num_mats; a.w.sctl[1] = 0; }
-    grid_barrier(kp);
-    radix_sort_phase(kp, a.w, 0, 64, reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
-    const int32_t* order = ld_cg_s32(a.w.sctl + 1) ? a.w.vals1 : a.w.vals0;
-    Problem* solos = const_cast<Problem*>(kp.solos);
-    for (int i = gtid(); i < a.num_mats; i += G) {
-      const int k = __ldcg(order + i);
-      Problem P;
-      P.node_base = a.node_off[k];
-      P.rp_base = a.node_off[k] + k;
-      P.ci_base = a.nnz_off[k];
-      P.o_base = a.node_off[k];
-      P.perm_base = a.node_off[k];
-      P.mat_n = (int)(a.node_off[k + 1] - a.node_off[k]);
-      P.pos0 = 0;
-      P.size = P.mat_n;
-      P.seed = (a.mode == RCM_START_FIXED && a.starts) ? a.starts[k] : (int)(uint32_t)__ldcg(a.pm_key + k);
-      P.flags = 1 | gl_flag;
-      P.pad = 0;
-      solos[i] = P;
-    }
-    if (gtid() == 0) kp.ctl->n_solo = a.num_mats;
-  } else {
-    int seed = a.mode == RCM_START_FIXED ? a.start : (int)(uint32_t)__ldcg(&kp.ctl->minkey);
-    if (a.mode == RCM_START_PSEUDO_PERIPHERAL && !a.solo) seed = gl_phase(kp, a.w, a.n, seed, sh);
-    if (gtid() == 0) {
-      Problem P;
-      P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
-      P.mat_n = a.n; P.pos0 = 0; P.size = a.n; P.seed = seed; P.pad = 0;
-      if (a.solo) { P.flags = 1 | gl_flag; const_cast<Problem*>(kp.solos)[0] = P; kp.ctl->n_solo = 1; }
-      else { P.flags = 0; const_cast<Problem*>(kp.chains)[0] = P; kp.ctl->n_chain = 1; }
-    }
+  int seed = a.mode == RCM_START_FIXED ? a.start : (int)(uint32_t)__ldcg(&kp.ctl->minkey);
+  if (a.mode == RCM_START_PSEUDO_PERIPHERAL) seed = gl_phase(kp, a.w, a.n, seed, sh);
+  if (gtid() == 0) {
+    Problem P;
+    P.node_base = 0; P.rp_base = 0; P.ci_base = 0; P.o_base = 0; P.perm_base = 0;
+    P.mat_n = a.n; P.pos0 = 0; P.size = a.n; P.seed = seed; P.pad = 0;
+    P.flags = 0;
+    const_cast<Problem*>(kp.chains)[0] = P;
+    kp.ctl->n_chain = 1;
   }
   grid_barrier(kp);
   stamp(kp, 2);
@@ -254,7 +184,7 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
   grid_barrier(kp);
   stamp(kp, 3);
   // ---- phase 4: components left over by the chain-first pass (a13)
-  if (!a.batched && !a.solo && ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
+  if (ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
     cc_phase(kp, a, sm, sh);
     schedule_phase<kMB>(kp, a, sm, sh, sh2);
     grid_barrier(kp);

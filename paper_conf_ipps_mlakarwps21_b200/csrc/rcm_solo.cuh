@@ -1,0 +1,795 @@
+// rcm_solo.cuh -- the batched / small-graph path: one matrix (or one small
+// graph) per thread block, many blocks per SM, no inter-block signalling.
+//
+// Inside one block the batches of the paper's method (Alg. 5) run
+// one after the other, so the speculation / rediscovery / chain of the
+// multi-block path is not needed: when a batch starts, every earlier batch is
+// complete.  What remains of a batch is:
+//   parents    the next nP <= B_s nodes of the CM order o, whose summed
+//              valence fits the T edge slots; held with their row
+//              start and valence in a shared-memory ring, so a batch does not
+//              re-read o[] or row_ptr for its parents;
+//   discover   every edge (p, c) of the batch with c not yet placed (a
+//              shared-memory VISITED BITMAP, one bit per node of the matrix,
+//              replaces the owner-word prefilter of the multi-block path)
+//              inserts (c, edge slot e) into a shared-memory CLAIM TABLE that
+//              keeps, per child c, the minimum edge slot.  Edge slots are laid
+//              out parent by parent, so the minimum slot is the earliest parent
+//              in o (Alg. 1 ln 8-12: the first parent to see c claims it,
+//              P:L202-212) and, within one parent, the first of duplicate
+//              entries (C-8).  The child's valence r[c+1]-r[c] and row
+//              start are loaded while the claims are inserted;
+//   sort       the winners of each parent, by (valence, id) (C-1);
+//   output     at the next positions of o, written reversed into perm
+//              and appended to the ring as future parents.
+// There is no global atomic and no owner word: per batch two dependent global
+// round trips remain (the batch's columns, then the children's row_ptr).
+//
+// Seeds follow C-6 (min (valence, id) over the unplaced nodes, found with a
+// cursor that only moves forward because that minimum never decreases), FIXED
+// starts, and the GL finder (C-5) by a block-level BFS.  A parent
+// whose valence exceeds T is processed in chunks of T edges; its
+// children are sorted in plan-owned HBM scratch by a block radix sort.
+// Matrices above the shared-memory bitmap capacity keep their bitmaps in HBM
+// (same code, global atomics).  DESIGN.md §2.6.
+#pragma once
+#include "rcm_batch.cuh"
+
+namespace rcm {
+
+#ifndef RCM_SOLO_NT
+#define RCM_SOLO_NT 256
+#endif
+#ifndef RCM_SOLO_U
+#define RCM_SOLO_U 4
+#endif
+#ifndef RCM_SOLO_Q
+#define RCM_SOLO_Q 512
+#endif
+constexpr int kSoloNT = RCM_SOLO_NT;                // threads per block
+constexpr int kSoloNW = kSoloNT / 32;
+constexpr int kSoloU = RCM_SOLO_U;                  // edge slots per thread per batch
+constexpr int kSoloT = kSoloNT * kSoloU;            // T: edge slots of a batch
+constexpr int kSoloH = 2 * kSoloT;                  // claim-table slots (power of two)
+constexpr int kSoloHBits = __builtin_ctz(kSoloH);
+constexpr int kSoloQ = RCM_SOLO_Q;                  // ring of pending parents (power of two)
+constexpr int kSoloNMax = (1 << 17) - 1;            // shared-memory bitmap capacity (nodes)
+constexpr int kSoloVisW = (kSoloNMax >> 5) + 1;     // bitmap words
+static_assert(kSoloT <= 32767 && (kSoloH & (kSoloH - 1)) == 0 && kSoloHBits <= 15, "claim table packing");
+static_assert((kSoloQ & (kSoloQ - 1)) == 0 && kSoloQ >= 256, "ring size");
+constexpr uint32_t kEmpty32 = 0xFFFFFFFFu;          // (c:17 | e:15) never reaches it: c < 2^17 - 1
+constexpr int kSoloGrp = 256;                       // output-group ring (stats only)
+
+// Arguments of the solo kernels (one launch of k_solo_order + one of k_solo).
+struct SoloArgs {
+  const int32_t* row_ptr;     // batched: per matrix n_k + 1 local offsets, concatenated
+  const int32_t* col_idx;     // local column ids
+  int32_t* perm;              // output (new -> old, local ids)
+  int32_t* iperm;             // nullable (single graph only)
+  const int64_t* node_off;    // nullable: single graph of n nodes / nnz entries
+  const int64_t* nnz_off;
+  const int32_t* starts;      // nullable: per-matrix FIXED starts
+  int32_t* order;             // matrix processing order (largest first)
+  uint32_t* gvis;             // HBM bitmaps for matrices above kSoloNMax: 2 x gvis_words
+  long long gvis_words;
+  unsigned long long* spill;  // oversize scratch: keys [0, cap), radix temp [cap, 2 cap)
+  long long spill_cap;
+  Ctl* ctl;
+  Stats* stats;
+  int num_mats;
+  int n;                      // single graph
+  long long nnz;
+  int mode;
+  int start;                  // single graph FIXED start
+  int validate;
+  int collect_stats;
+  int flags;
+  int BS;                     // B_s (<= kSoloNT)
+};
+
+// Shared-memory layout (bytes), dynamic.
+constexpr size_t kSoOffVis = 0;
+constexpr size_t kSoOffRing = kSoOffVis + 4 * (size_t)kSoloVisW;
+constexpr size_t kSoOffPar = kSoOffRing + 12 * (size_t)kSoloQ;                 // 5 int arrays of kSoloNT + 1
+constexpr size_t kSoOffLpof = kSoOffPar + 5 * 4 * (size_t)(kSoloNT + 1) + 12;
+constexpr size_t kSoOffCand = (kSoOffLpof + 2 * (size_t)kSoloT + 15) & ~size_t(15);
+constexpr size_t kSoOffHash = kSoOffCand + 8 * (size_t)kSoloT;
+constexpr size_t kSoOffRsv = kSoOffHash + 4 * (size_t)kSoloH;                  // big matrices: 8 B entries over hash+rsv
+constexpr size_t kSoloSmem = kSoOffRsv + 4 * (size_t)kSoloH;
+static_assert(kSoloSmem - kSoOffLpof >= 4 * (size_t)kSoloVisW, "GL bitmap overlays lpof..rsv");
+
+struct SoloSh {
+  int32_t wtmp[kSoloNW + 1];
+  long long wtmpll[kSoloNW + 1];
+  unsigned long long wtmp64[kSoloNW + 1];
+  int32_t k, pos, written, rhi, nP, E, cnt, tail, found, big_n;
+  int32_t cur_deg, cur_id, bad;
+  unsigned long long minkey;
+  int32_t big_list[kSoloNT];
+  long long st_exec, st_comp, st_over, st_claim, st_comb;
+  // start positions of the pending output groups (one per batch), for the
+  // work-aggregation counter: a batch whose parents span several groups
+  // combines the outputs of several earlier batches
+  int32_t grp[kSoloGrp];
+  int32_t grp_h, grp_t;
+};
+
+// Matrix geometry.
+struct SoloMat {
+  const int32_t* rp;   // local row_ptr (n + 1)
+  const int32_t* col;  // local columns (add rp values)
+  int32_t* perm;       // local perm (n)
+  long long node_base;
+  int n;
+  int nnz;
+  uint32_t* vis;       // placed bitmap (smem or HBM)
+  uint32_t* bvis;      // GL BFS bitmap (smem overlay or HBM)
+  bool gmem;           // bitmaps in HBM
+};
+
+__device__ __forceinline__ uint8_t* so_base() { return rcm_dsm; }
+__device__ __forceinline__ int32_t* so_ring_v() { return reinterpret_cast<int32_t*>(so_base() + kSoOffRing); }
+__device__ __forceinline__ int32_t* so_ring_rs() { return so_ring_v() + kSoloQ; }
+__device__ __forceinline__ int32_t* so_ring_d() { return so_ring_v() + 2 * kSoloQ; }
+__device__ __forceinline__ int32_t* so_p_v() { return reinterpret_cast<int32_t*>(so_base() + kSoOffPar); }
+__device__ __forceinline__ int32_t* so_p_rs() { return so_p_v() + (kSoloNT + 1); }
+__device__ __forceinline__ int32_t* so_p_eo() { return so_p_v() + 2 * (kSoloNT + 1); }
+__device__ __forceinline__ int32_t* so_p_cnt() { return so_p_v() + 3 * (kSoloNT + 1); }
+__device__ __forceinline__ int32_t* so_p_pfx() { return so_p_v() + 4 * (kSoloNT + 1); }
+__device__ __forceinline__ uint16_t* so_lpof() { return reinterpret_cast<uint16_t*>(so_base() + kSoOffLpof); }
+__device__ __forceinline__ unsigned long long* so_cand() {
+  return reinterpret_cast<unsigned long long*>(so_base() + kSoOffCand);
+}
+__device__ __forceinline__ uint32_t* so_hash() { return reinterpret_cast<uint32_t*>(so_base() + kSoOffHash); }
+__device__ __forceinline__ unsigned long long* so_hash64() {
+  return reinterpret_cast<unsigned long long*>(so_base() + kSoOffHash);
+}
+__device__ __forceinline__ int32_t* so_rsv() { return reinterpret_cast<int32_t*>(so_base() + kSoOffRsv); }
+
+// ------------------------------------------------------------- block helpers
+template <typename T>
+__device__ __forceinline__ T so_scan(T v, T* wtmp, T& total) {   // exclusive, kSoloNT threads
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  T x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T y = __shfl_up_sync(0xffffffffu, x, d);
+    if (lane >= d) x += y;
+  }
+  if (lane == 31) wtmp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    T w = lane < kSoloNW ? wtmp[lane] : T(0);
+    T s = w;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      T y = __shfl_up_sync(0xffffffffu, s, d);
+      if (lane >= d) s += y;
+    }
+    if (lane < kSoloNW) wtmp[lane] = s - w;
+    if (lane == kSoloNW - 1) wtmp[kSoloNW] = s;
+  }
+  __syncthreads();
+  const T r = wtmp[wid] + x - v;
+  total = wtmp[kSoloNW];
+  __syncthreads();
+  return r;
+}
+
+__device__ __forceinline__ unsigned long long so_min_u64(unsigned long long v, SoloSh& sh) {
+  v = warp_min_u64(v);
+  if ((threadIdx.x & 31) == 0) sh.wtmp64[threadIdx.x >> 5] = v;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    unsigned long long b = threadIdx.x < kSoloNW ? sh.wtmp64[threadIdx.x] : kKeyMax;
+    b = warp_min_u64(b);
+    if (threadIdx.x == 0) sh.minkey = b;
+  }
+  __syncthreads();
+  const unsigned long long r = sh.minkey;
+  __syncthreads();
+  return r;
+}
+
+__device__ __forceinline__ bool so_test(const SoloMat& M, int v) {
+  const uint32_t w = M.gmem ? __ldcg(M.vis + (v >> 5)) : M.vis[v >> 5];
+  return (w >> (v & 31)) & 1u;
+}
+__device__ __forceinline__ void so_set(const SoloMat& M, uint32_t* bits, int v) {
+  atomicOr(bits + (v >> 5), 1u << (v & 31));
+}
+// test-and-set, true if this call set the bit
+__device__ __forceinline__ bool so_claim_bit(uint32_t* bits, int v) {
+  const uint32_t b = 1u << (v & 31);
+  return !(atomicOr(bits + (v >> 5), b) & b);
+}
+
+__device__ __forceinline__ void so_zero_bits(uint32_t* bits, int n) {
+  for (int i = threadIdx.x; i < (n >> 5) + 1; i += kSoloNT) bits[i] = 0u;
+}
+
+__device__ __forceinline__ uint32_t so_hslot(uint32_t c) { return (c * 2654435761u) >> (32 - kSoloHBits); }
+
+// Insert claim (c, e) into the table: per child the minimum edge slot (small
+// matrices: one 32-bit word c:17 | e:15; large: c:32 | e:32).  Returns the slot.
+template <bool kBig>
+__device__ __forceinline__ int so_claim(uint32_t c, uint32_t e) {
+  uint32_t s = so_hslot(c);
+  if constexpr (!kBig) {
+    volatile uint32_t* h = so_hash();
+    const uint32_t want = (c << 15) | e;
+    for (;;) {
+      uint32_t cur = h[s];
+      if (cur == kEmpty32) {
+        cur = atomicCAS(const_cast<uint32_t*>(h) + s, kEmpty32, want);
+        if (cur == kEmpty32) return (int)s;
+      }
+      if ((cur >> 15) == c) { atomicMin(const_cast<uint32_t*>(h) + s, want); return (int)s; }
+      s = (s + 1) & (kSoloH - 1);
+    }
+  } else {
+    volatile unsigned long long* h = so_hash64();
+    const unsigned long long want = ((unsigned long long)c << 32) | e;
+    for (;;) {
+      unsigned long long cur = h[s];
+      if (cur == kKeyMax) {
+        cur = atomicCAS(const_cast<unsigned long long*>(h) + s, kKeyMax, want);
+        if (cur == kKeyMax) return (int)s;
+      }
+      if ((uint32_t)(cur >> 32) == c) { atomicMin(const_cast<unsigned long long*>(h) + s, want); return (int)s; }
+      s = (s + 1) & (kSoloH - 1);
+    }
+  }
+}
+template <bool kBig>
+__device__ __forceinline__ bool so_won(int s, uint32_t c, uint32_t e) {
+  if constexpr (!kBig) return so_hash()[s] == ((c << 15) | e);
+  else return so_hash64()[s] == (((unsigned long long)c << 32) | e);
+}
+template <bool kBig>
+__device__ __forceinline__ void so_unclaim(int s) {
+  if constexpr (!kBig) so_hash()[s] = kEmpty32;
+  else so_hash64()[s] = kKeyMax;
+}
+
+// Every claim-table slot empty (after the GL bitmap or the radix scratch
+// overlaid the table).
+template <bool kBig>
+__device__ __forceinline__ void so_hash_reset() {
+  if constexpr (!kBig) for (int i = threadIdx.x; i < kSoloH; i += kSoloNT) so_hash()[i] = kEmpty32;
+  else for (int i = threadIdx.x; i < kSoloH; i += kSoloNT) so_hash64()[i] = kKeyMax;
+  __syncthreads();
+}
+
+// Stable LSD radix sort (8-bit digits, constant digits skipped) of a[0..n) in
+// HBM by one block, temp tmp[0..n).  Used for an oversize parent's children.
+static __device__ void so_radix_sort_global(unsigned long long* a, unsigned long long* tmp, int n, SoloSh& sh) {
+  if (n <= 1) return;
+  int32_t* off = reinterpret_cast<int32_t*>(so_cand());       // 256 digit offsets
+  int32_t* wcnt = off + 256;                                  // kSoloNW x 256
+  const unsigned long long first = __ldcg(a);
+  unsigned long long diff = 0;
+  for (int i = threadIdx.x; i < n; i += kSoloNT) diff |= __ldcg(a + i) ^ first;
+  diff = ~so_min_u64(~diff, sh);                              // block OR
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const unsigned lt = (1u << lane) - 1;
+  unsigned long long* src = a;
+  unsigned long long* dst = tmp;
+  for (int shift = 0; shift < 64; shift += 8) {
+    if (((diff >> shift) & 0xffull) == 0) continue;
+    for (int i = threadIdx.x; i < 256; i += kSoloNT) off[i] = 0;
+    __syncthreads();
+    for (int i = threadIdx.x; i < n; i += kSoloNT) atomicAdd(&off[(__ldcg(src + i) >> shift) & 0xff], 1);
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      int v[8], s = 0;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) { v[j] = off[threadIdx.x * 8 + j]; s += v[j]; }
+      int x = s;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) { int y = __shfl_up_sync(0xffffffffu, x, d); if (threadIdx.x >= d) x += y; }
+      int run = x - s;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) { off[threadIdx.x * 8 + j] = run; run += v[j]; }
+    }
+    __syncthreads();
+    for (int base = 0; base < n; base += kSoloNT) {
+      const int i = base + threadIdx.x;
+      const bool valid = i < n;
+      const unsigned long long k = valid ? __ldcg(src + i) : 0ull;
+      const int d = valid ? (int)((k >> shift) & 0xff) : 256;
+      const unsigned peers = __match_any_sync(0xffffffffu, d);
+      const int rank = __popc(peers & lt);
+      for (int j = threadIdx.x; j < kSoloNW * 256; j += kSoloNT) wcnt[j] = 0;
+      __syncthreads();
+      if (valid && rank == 0) wcnt[wid * 256 + d] = __popc(peers);
+      __syncthreads();
+      for (int dg = threadIdx.x; dg < 256; dg += kSoloNT) {
+        int run = off[dg];
+        for (int w = 0; w < kSoloNW; ++w) { const int c = wcnt[w * 256 + dg]; wcnt[w * 256 + dg] = run; run += c; }
+        off[dg] = run;
+      }
+      __syncthreads();
+      if (valid) dst[wcnt[wid * 256 + d] + rank] = k;
+      __syncthreads();
+    }
+    unsigned long long* t = src; src = dst; dst = t;
+  }
+  if (src != a)
+    for (int i = threadIdx.x; i < n; i += kSoloNT) a[i] = __ldcg(src + i);
+  __syncthreads();
+}
+
+// --------------------------------------------------------------- seeds / GL
+// Valence of local node v.
+__device__ __forceinline__ int so_deg(const SoloMat& M, int v) { return __ldg(M.rp + v + 1) - __ldg(M.rp + v); }
+
+// Block-level BFS over the (wholly unplaced) component of r for the GL finder:
+// the queue lives in the not-yet-written part of perm, visited bits in M.bvis.
+// Returns the number of levels; *minkey = min (valence, id) of the last level.
+static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long long* minkey, SoloSh& sh) {
+  int32_t* q = M.perm;                        // entries [0, n - written) are free
+  so_zero_bits(M.bvis, M.n);
+  __syncthreads();
+  if (threadIdx.x == 0) { q[0] = r; so_claim_bit(M.bvis, r); sh.tail = 1; }
+  __syncthreads();
+  int head = 0, tail = 1, levels = 1;
+  for (;;) {
+    for (int i = head + threadIdx.x; i < tail; i += kSoloNT) {
+      const int p = __ldcg(q + i);
+      for (int e = __ldg(M.rp + p), ee = __ldg(M.rp + p + 1); e < ee; ++e) {
+        const int c = __ldg(M.col + e);
+        if (so_claim_bit(M.bvis, c)) q[atomicAdd(&sh.tail, 1)] = c;
+      }
+    }
+    __syncthreads();
+    const int nt = sh.tail;
+    __syncthreads();
+    if (nt == tail) break;
+    head = tail;
+    tail = nt;
+    ++levels;
+  }
+  unsigned long long best = kKeyMax;
+  for (int i = head + threadIdx.x; i < tail; i += kSoloNT) {
+    const int v = __ldcg(q + i);
+    const unsigned long long k = ((unsigned long long)(uint32_t)so_deg(M, v) << 32) | (uint32_t)v;
+    best = k < best ? k : best;
+  }
+  *minkey = so_min_u64(best, sh);
+  return levels;
+}
+
+// GL finder (C-5): BFS from r, next root = min (valence, id) of the
+// last level, repeat while the level count grows, return the last root.
+static __device__ int so_gl(const SoloMat& M, int written, int r, SoloSh& sh) {
+  unsigned long long key;
+  int nl = so_bfs(M, written, r, &key, sh);
+  int x = (int)(uint32_t)key;
+  for (;;) {
+    const int nx = so_bfs(M, written, x, &key, sh);
+    if (nx <= nl) break;
+    nl = nx;
+    x = (int)(uint32_t)key;
+  }
+  if (!M.gmem) so_hash_reset<false>();   // the BFS bitmap overlaid the claim table
+  return x;
+}
+
+// Next C-6 seed: min (valence, id) over the unplaced nodes.  The minimum never
+// decreases as nodes get placed, so a cursor (cur_deg, cur_id) scans forward:
+// first the ids after cur_id with valence cur_deg, then the next larger
+// valence present.  O(n) per distinct valence, not per component.
+static __device__ int so_next_seed(const SoloMat& M, SoloSh& sh) {
+  for (;;) {
+    const int d = sh.cur_deg;
+    for (int base = sh.cur_id + 1; base < M.n; base += kSoloNT) {
+      const int v = base + threadIdx.x;
+      const bool f = v < M.n && !so_test(M, v) && so_deg(M, v) == d;
+      if (threadIdx.x == 0) sh.found = 0x7fffffff;
+      __syncthreads();
+      if (f) atomicMin(&sh.found, v);
+      __syncthreads();
+      const int s = sh.found;
+      __syncthreads();
+      if (s != 0x7fffffff) {
+        if (threadIdx.x == 0) sh.cur_id = s;
+        __syncthreads();
+        return s;
+      }
+    }
+    unsigned long long best = kKeyMax;   // smallest valence above d among unplaced
+    for (int v = threadIdx.x; v < M.n; v += kSoloNT) {
+      if (so_test(M, v)) continue;
+      const int dv = so_deg(M, v);
+      if (dv > d) {
+        const unsigned long long k = ((unsigned long long)(uint32_t)dv << 32) | (uint32_t)v;
+        best = k < best ? k : best;
+      }
+    }
+    best = so_min_u64(best, sh);
+    if (best == kKeyMax) return -1;
+    if (threadIdx.x == 0) { sh.cur_deg = (int)(best >> 32); sh.cur_id = (int)(uint32_t)best; }
+    __syncthreads();
+    return (int)(uint32_t)best;
+  }
+}
+
+// Place a root at position q (thread 0): perm, iperm, placed bit, ring.
+__device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int s, int q) {
+  M.perm[M.n - 1 - q] = s;
+  if (a.iperm) a.iperm[M.node_base + s] = M.n - 1 - q;
+  so_set(M, M.vis, s);
+  if (sh.rhi == q) {   // ring contiguous up to the output end
+    so_ring_v()[q & (kSoloQ - 1)] = s;
+    so_ring_rs()[q & (kSoloQ - 1)] = __ldg(M.rp + s);
+    so_ring_d()[q & (kSoloQ - 1)] = so_deg(M, s);
+    sh.rhi = q + 1;
+  }
+}
+
+// ------------------------------------------------------------ validation
+// validate >= 1: r[0] = 0, non-decreasing, r[n] = nnz, 0 <= col < n;
+// validate == 2: every (u, c) has (c, u) (binary search in sorted rows, linear
+// scan otherwise).  Returns true if the matrix is well formed.
+static __device__ bool so_validate(const SoloArgs& a, const SoloMat& M, SoloSh& sh) {
+  int bad = 0;
+  if (threadIdx.x == 0) bad = (__ldg(M.rp) != 0) || (__ldg(M.rp + M.n) != M.nnz);
+  for (int v = threadIdx.x; v < M.n; v += kSoloNT) bad |= __ldg(M.rp + v + 1) < __ldg(M.rp + v);
+  bad = __syncthreads_or(bad);
+  if (!bad)
+    for (int i = threadIdx.x; i < M.nnz; i += kSoloNT) {
+      const int c = __ldg(M.col + i);
+      bad |= (c < 0 || c >= M.n);
+    }
+  bad = __syncthreads_or(bad);
+  if (bad) {
+    if (threadIdx.x == 0) atomicCAS(&a.ctl->status, 0, ST_BAD_CSR);
+    return false;
+  }
+  if (a.validate < 2) return true;
+  int asym = 0;
+  for (int u = threadIdx.x; u < M.n && !asym; u += kSoloNT) {   // thread per row
+    for (int e = __ldg(M.rp + u), re = __ldg(M.rp + u + 1); e < re && !asym; ++e) {
+      const int c = __ldg(M.col + e);
+      int lo = __ldg(M.rp + c), hi = __ldg(M.rp + c + 1) - 1;
+      const int b0 = lo, b1 = hi;
+      bool found = false;
+      while (lo <= hi) {   // sorted row: O(log deg)
+        const int mid = (lo + hi) >> 1;
+        const int x = __ldg(M.col + mid);
+        if (x == u) { found = true; break; }
+        if (x < u) lo = mid + 1; else hi = mid - 1;
+      }
+      for (int f = b0; f <= b1 && !found; ++f) found = __ldg(M.col + f) == u;   // unsorted row
+      asym |= !found;
+    }
+  }
+  asym = __syncthreads_or(asym);
+  if (asym && threadIdx.x == 0) atomicCAS(&a.ctl->status, 0, ST_NOT_SYM);
+  return !asym;
+}
+
+// ---------------------------------------------------------------- batches
+// Sort each parent's winners by (valence, id): <= 16 by one thread, else one warp.
+static __device__ void so_sort_segments(int nP, SoloSh& sh) {
+  if (threadIdx.x == 0) sh.big_n = 0;
+  __syncthreads();
+  unsigned long long* cand = so_cand();
+  for (int lp = threadIdx.x; lp < nP; lp += kSoloNT) {
+    const int n = so_p_cnt()[lp];
+    if (n <= 1) continue;
+    unsigned long long* a = cand + so_p_eo()[lp];
+    if (n <= 16) {
+      for (int i = 1; i < n; ++i) {
+        const unsigned long long x = a[i];
+        int j = i - 1;
+        while (j >= 0 && a[j] > x) { a[j + 1] = a[j]; --j; }
+        a[j + 1] = x;
+      }
+    } else {
+      sh.big_list[atomicAdd(&sh.big_n, 1)] = lp;
+    }
+  }
+  __syncthreads();
+  const int nbig = sh.big_n;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  for (int b = wid; b < nbig; b += kSoloNW) {
+    const int lp = sh.big_list[b];
+    bitonic_sort_flip(cand + so_p_eo()[lp], so_p_cnt()[lp], lane, 32, [] { __syncwarp(); });
+  }
+  __syncthreads();
+}
+
+// One batch of parents [pos, pos + nP) whose edges fit the T slots.
+template <bool kBig>
+static __device__ void so_batch(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int nP) {
+  const int E = so_p_eo()[nP];
+  const int pos = sh.pos, written = sh.written;
+  // edge slot -> local parent, one warp per parent
+  {
+    const int lane = threadIdx.x & 31;
+    for (int lp = threadIdx.x >> 5; lp < nP; lp += kSoloNW) {
+      const int eb = so_p_eo()[lp], ee = so_p_eo()[lp + 1];
+      for (int j = eb + lane; j < ee; j += 32) so_lpof()[j] = (uint16_t)lp;
+    }
+  }
+  __syncthreads();
+  // discover: columns, placed test, claims; child row_ptr loads in flight
+  int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
+#pragma unroll
+  for (int u = 0; u < kSoloU; ++u) {
+    const int e = threadIdx.x + u * kSoloNT;
+    cc[u] = -1;
+    if (e < E) {
+      const int lp = so_lpof()[e];
+      cc[u] = __ldg(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < kSoloU; ++u) {
+    if (cc[u] >= 0 && so_test(M, cc[u])) cc[u] = -1;   // placed (self-loops included)
+    if (cc[u] >= 0) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+  }
+#pragma unroll
+  for (int u = 0; u < kSoloU; ++u)
+    if (cc[u] >= 0) slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT));
+  __syncthreads();
+  // winners: the minimum edge slot per child = the earliest parent
+  int won = 0;
+#pragma unroll
+  for (int u = 0; u < kSoloU; ++u) {
+    const int e = threadIdx.x + u * kSoloNT;
+    if (cc[u] >= 0 && so_won<kBig>(slot[u], (uint32_t)cc[u], (uint32_t)e)) {
+      const int lp = so_lpof()[e];
+      const int idx = atomicAdd(&so_p_cnt()[lp], 1);
+      const unsigned long long d = (unsigned long long)(uint32_t)(cre[u] - crs[u]);
+      unsigned long long key;
+      if constexpr (!kBig) {
+        so_rsv()[slot[u]] = crs[u];
+        key = (d << 32) | ((unsigned long long)(uint32_t)cc[u] << 15) | (uint32_t)slot[u];
+      } else {
+        key = (d << 32) | (uint32_t)cc[u];
+      }
+      so_cand()[so_p_eo()[lp] + idx] = key;
+      so_set(M, M.vis, cc[u]);
+      ++won;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int u = 0; u < kSoloU; ++u)
+    if (cc[u] >= 0) so_unclaim<kBig>(slot[u]);   // (table reads are done)
+  if (!(a.flags & F_NO_SORT)) so_sort_segments(nP, sh);
+  // output positions: exclusive prefix of the per-parent counts
+  int tot;
+  const int mycnt = threadIdx.x < nP ? so_p_cnt()[threadIdx.x] : 0;
+  const int pf = so_scan<int32_t>(mycnt, sh.wtmp, tot);
+  if (threadIdx.x < nP) so_p_pfx()[threadIdx.x] = pf;
+  __syncthreads();
+  const int pos_new = pos + nP;
+  const bool ring_ok = !kBig && sh.rhi == written;
+  const int last = M.n - 1;
+  for (int i = threadIdx.x; i < E; i += kSoloNT) {
+    const int lp = so_lpof()[i];
+    const int j = i - so_p_eo()[lp];
+    if (j >= so_p_cnt()[lp]) continue;
+    const unsigned long long key = so_cand()[i];
+    const int q = written + so_p_pfx()[lp] + j;
+    int c;
+    if constexpr (!kBig) c = (int)((key >> 15) & 0x1ffffu);
+    else c = (int)(uint32_t)key;
+    M.perm[last - q] = c;
+    if (a.iperm) a.iperm[M.node_base + c] = last - q;
+    if constexpr (!kBig) {
+      if (ring_ok && q < pos_new + kSoloQ) {
+        so_ring_v()[q & (kSoloQ - 1)] = c;
+        so_ring_rs()[q & (kSoloQ - 1)] = so_rsv()[key & 0x7fffu];
+        so_ring_d()[q & (kSoloQ - 1)] = (int)(key >> 32);
+      }
+    }
+  }
+  if (a.collect_stats && won) atomicAdd(reinterpret_cast<unsigned long long*>(&sh.st_claim), (unsigned long long)won);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    sh.pos = pos_new;
+    sh.written = written + tot;
+    if (ring_ok) sh.rhi = min(written + tot, pos_new + kSoloQ);
+    ++sh.st_exec;
+    if (a.collect_stats && tot > 0 && sh.grp_t - sh.grp_h < kSoloGrp) sh.grp[(sh.grp_t++) & (kSoloGrp - 1)] = written;
+  }
+  __syncthreads();
+}
+
+// A parent whose valence exceeds T: its row in chunks of T edge
+// slots, winners to HBM scratch, one block radix sort by (valence, id).
+template <bool kBig>
+static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int rs, int D) {
+  unsigned long long* keys = a.spill + M.node_base;
+  if (threadIdx.x == 0) sh.cnt = 0;
+  __syncthreads();
+  for (int c0 = 0; c0 < D; c0 += kSoloT) {
+    int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      const int e = c0 + threadIdx.x + u * kSoloNT;
+      cc[u] = e < D ? __ldg(M.col + rs + e) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      if (cc[u] >= 0 && so_test(M, cc[u])) cc[u] = -1;
+      if (cc[u] >= 0) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+    }
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u)
+      if (cc[u] >= 0) slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT));
+    __syncthreads();
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      if (cc[u] >= 0 && so_won<kBig>(slot[u], (uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT))) {
+        const int idx = atomicAdd(&sh.cnt, 1);
+        keys[idx] = ((unsigned long long)(uint32_t)(cre[u] - crs[u]) << 32) | (uint32_t)cc[u];
+        so_set(M, M.vis, cc[u]);
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u)
+      if (cc[u] >= 0) so_unclaim<kBig>(slot[u]);
+    __syncthreads();
+  }
+  const int C = sh.cnt;
+  if (!(a.flags & F_NO_SORT)) {
+    so_radix_sort_global(keys, a.spill + a.spill_cap + M.node_base, C, sh);
+    so_hash_reset<kBig>();   // the sort's digit counters overlaid the table
+  }
+  const int written = sh.written, last = M.n - 1;
+  for (int i = threadIdx.x; i < C; i += kSoloNT) {
+    const int c = (int)(uint32_t)__ldcg(keys + i);
+    M.perm[last - written - i] = c;
+    if (a.iperm) a.iperm[M.node_base + c] = last - written - i;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    sh.pos += 1;
+    sh.written = written + C;   // the ring is not extended: these parents are refilled from perm
+    ++sh.st_exec;
+    ++sh.st_over;
+  }
+  __syncthreads();
+}
+
+// Choose the next batch: refill the ring from perm when it runs low, then the
+// longest prefix of [pos, rhi) (at most B_s) whose valences fit T.
+template <bool kBig>
+static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh) {
+  const int pos = sh.pos, written = sh.written;
+  int rhi = sh.rhi;
+  const int last = M.n - 1;
+  if (kBig || (rhi < written && rhi - pos < a.BS)) {
+    const int lo = kBig ? pos : max(rhi, pos);
+    const int hi = min(written, pos + kSoloQ);
+    for (int q = lo + threadIdx.x; q < hi; q += kSoloNT) {
+      const int v = __ldcg(M.perm + last - q);
+      const int r0 = __ldg(M.rp + v);
+      so_ring_v()[q & (kSoloQ - 1)] = v;
+      so_ring_rs()[q & (kSoloQ - 1)] = r0;
+      so_ring_d()[q & (kSoloQ - 1)] = __ldg(M.rp + v + 1) - r0;
+    }
+    rhi = hi;
+    __syncthreads();
+    if (threadIdx.x == 0 && !kBig) sh.rhi = hi;   // big matrices: the ring is only a staging buffer
+  }
+  const int avail = min(a.BS, rhi - pos);
+  const int t = threadIdx.x;
+  const int d = t < avail ? so_ring_d()[(pos + t) & (kSoloQ - 1)] : 0;
+  int tot;
+  const int eo = so_scan<int32_t>(d, sh.wtmp, tot);
+  const bool fit = t < avail && eo + d <= kSoloT;
+  if (fit) {
+    so_p_v()[t] = so_ring_v()[(pos + t) & (kSoloQ - 1)];
+    so_p_rs()[t] = so_ring_rs()[(pos + t) & (kSoloQ - 1)];
+    so_p_eo()[t] = eo;
+    so_p_cnt()[t] = 0;
+  }
+  const int nP = __syncthreads_count(fit);
+  if (nP == 0) {   // the first parent alone exceeds T
+    so_oversize<kBig>(a, M, sh, so_ring_rs()[pos & (kSoloQ - 1)], so_ring_d()[pos & (kSoloQ - 1)]);
+    return;
+  }
+  if (t == nP - 1) so_p_eo()[nP] = eo + d;
+  if (t == 0 && a.collect_stats) {   // does this batch combine several earlier outputs?
+    while (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] <= pos) ++sh.grp_h;
+    if (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] < pos + nP) ++sh.st_comb;
+  }
+  __syncthreads();
+  so_batch<kBig>(a, M, sh, nP);
+}
+
+template <bool kBig>
+static __device__ void so_traverse(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int seed) {
+  if (threadIdx.x == 0) {
+    sh.pos = 0; sh.written = 0; sh.rhi = kBig ? -1 : 0;
+    sh.grp_h = sh.grp_t = 0;
+    so_place_root(a, M, sh, seed, 0);
+    sh.written = 1;
+    ++sh.st_comp;
+  }
+  __syncthreads();
+  for (;;) {
+    if (sh.pos == sh.written) {   // component exhausted (C-6)
+      if (sh.written >= M.n) break;
+      int s = so_next_seed(M, sh);
+      if (s < 0) { if (threadIdx.x == 0) atomicCAS(&a.ctl->status, 0, ST_BAD_CSR); break; }
+      if (a.mode == RCM_START_PSEUDO_PERIPHERAL) s = so_gl(M, sh.written, s, sh);
+      if (threadIdx.x == 0) {
+        so_place_root(a, M, sh, s, sh.written);
+        sh.written += 1;
+        ++sh.st_comp;
+      }
+      __syncthreads();
+      continue;
+    }
+    so_step<kBig>(a, M, sh);
+  }
+}
+
+// One matrix: validation, seed (C-5 / C-6 / FIXED), traversal.
+static __device__ void so_matrix(const SoloArgs& a, int k, SoloSh& sh) {
+  SoloMat M;
+  long long rp_base = 0, ci_base = 0;
+  if (a.node_off) {
+    M.node_base = __ldg(a.node_off + k);
+    M.n = (int)(__ldg(a.node_off + k + 1) - M.node_base);
+    ci_base = __ldg(a.nnz_off + k);
+    M.nnz = (int)(__ldg(a.nnz_off + k + 1) - ci_base);
+    rp_base = M.node_base + k;
+  } else {
+    M.node_base = 0;
+    M.n = a.n;
+    M.nnz = (int)a.nnz;
+  }
+  if (M.n <= 0) return;
+  M.rp = a.row_ptr + rp_base;
+  M.col = a.col_idx + ci_base;
+  M.perm = a.perm + M.node_base;
+  M.gmem = M.n > kSoloNMax;
+  if (M.gmem) {
+    const long long w = (M.node_base >> 5) + k;
+    M.vis = a.gvis + w;
+    M.bvis = a.gvis + a.gvis_words + w;
+  } else {
+    M.vis = reinterpret_cast<uint32_t*>(so_base() + kSoOffVis);
+    M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffLpof);   // overlays the batch scratch
+  }
+  if (a.validate && !so_validate(a, M, sh)) return;
+  int seed;
+  if (a.mode == RCM_START_FIXED) seed = a.node_off ? (a.starts ? __ldg(a.starts + k) : 0) : a.start;
+  else seed = 0;
+  if (seed < 0 || seed >= M.n) {   // FIXED start out of range (checked always: ADVICE r1)
+    if (threadIdx.x == 0) atomicCAS(&a.ctl->status, 0, ST_BAD_CSR);
+    return;
+  }
+  // prologue: argmin (valence, id) -- the MIN_DEGREE seed and the C-6 cursor
+  unsigned long long best = kKeyMax;
+  for (int v = threadIdx.x; v < M.n; v += kSoloNT) {
+    const unsigned long long key = ((unsigned long long)(uint32_t)so_deg(M, v) << 32) | (uint32_t)v;
+    best = key < best ? key : best;
+  }
+  so_zero_bits(M.vis, M.n);
+  // claim table starts empty (every batch restores it)
+  if (!M.gmem) so_hash_reset<false>();
+  else so_hash_reset<true>();
+  best = so_min_u64(best, sh);
+  if (a.mode != RCM_START_FIXED) seed = (int)(uint32_t)best;
+  if (threadIdx.x == 0) {
+    sh.cur_deg = (int)(best >> 32);
+    sh.cur_id = a.mode == RCM_START_FIXED ? -1 : seed;
+  }
+  __syncthreads();
+  if (a.mode == RCM_START_PSEUDO_PERIPHERAL) seed = so_gl(M, 0, seed, sh);
+  if (M.gmem) so_traverse<true>(a, M, sh, seed);
+  else so_traverse<false>(a, M, sh, seed);
+}
+
+}  // namespace rcm

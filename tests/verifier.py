@@ -118,9 +118,12 @@ def verify_small(row_ptr, col_idx, perm, mode=1, start=0):
     return None
 
 
-def verify(row_ptr, col_idx, perm, mode=1, start=0, check_gl=True):
+def verify(row_ptr, col_idx, perm, mode=1, start=0, check_gl=True, check_sort=True):
     """Vectorised V0-V4 (numpy, O(n + nnz) except V4 with mode 2 which runs a
-    BFS per root).  Returns None if valid else the name of the failed check."""
+    BFS per root).  Returns None if valid else the name of the failed check.
+    check_sort=False skips V3: what is left (V0-V2, V4) characterises a BFS
+    order with first-discovery parents, the output of RCM_FLAG_NO_SORT
+    (P:L1253-1254 "disable sorting ... BFS")."""
     row_ptr = np.asarray(row_ptr, dtype=np.int64)
     col_idx = np.asarray(col_idx, dtype=np.int64)
     perm = np.asarray(perm, dtype=np.int64)
@@ -155,7 +158,7 @@ def verify(row_ptr, col_idx, perm, mode=1, start=0, check_gl=True):
     same = ppn[1:] == ppn[:-1]
     kprev = dn[:-1] * (n + 1) + vn[:-1]
     knext = dn[1:] * (n + 1) + vn[1:]
-    if np.any(same & (kprev >= knext)):
+    if check_sort and np.any(same & (kprev >= knext)):
         return "V3"
     # V4: suffix minimum of (deg, id) over o
     key = deg[o] * (n + 1) + o
