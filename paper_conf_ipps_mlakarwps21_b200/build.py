@@ -37,22 +37,29 @@ def _extra_defines() -> list:
         extra.append(f"-DRCM_DISC_U={os.environ['RCM_DISC_U']}")
     if os.environ.get("RCM_TRACE"):
         extra.append("-DRCM_TRACE")
+    for k in ("RCM_SOLO_U", "RCM_SOLO_Q", "RCM_SOLO_NT", "RCM_SOLO_MINB"):   # solo-path variants (sweeps)
+        if os.environ.get(k):
+            extra.append(f"-D{k}={os.environ[k]}")
     return extra
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    """nvcc -c of every translation unit in parallel, then one -shared link."""
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None) -> str:
+    """nvcc -c of every translation unit in parallel, then one -shared link.
+    `out`: an alternative library path (variant builds for A/B sweeps, loaded
+    with RCM_LIB=...; objects then go to a private directory)."""
+    lib = out or LIB
+    if not force and not out and not _stale():
         return LIB
-    os.makedirs(BUILD_DIR, exist_ok=True)
+    bdir = BUILD_DIR if not out else os.path.join(BUILD_DIR, os.path.basename(out) + ".obj")
+    os.makedirs(bdir, exist_ok=True)
     extra = _extra_defines()
     if verbose:
         extra = ["-Xptxas=-v", *extra]
-    jobs = [(os.path.join(BUILD_DIR, "rcm.o"), [os.path.join(CSRC, "rcm.cu")]),
-            (os.path.join(BUILD_DIR, "k_solo.o"), [os.path.join(CSRC, "k_solo.cu")]),
-            (os.path.join(BUILD_DIR, "k_probe.o"), [os.path.join(CSRC, "k_probe.cu")])]
+    jobs = [(os.path.join(bdir, "rcm.o"), [os.path.join(CSRC, "rcm.cu")]),
+            (os.path.join(bdir, "k_solo.o"), [os.path.join(CSRC, "k_solo.cu")]),
+            (os.path.join(bdir, "k_probe.o"), [os.path.join(CSRC, "k_probe.cu")])]
     for bps, mb in KMAIN_VARIANTS:
-        jobs.append((os.path.join(BUILD_DIR, f"k_main_{bps}_{mb}.o"),
+        jobs.append((os.path.join(bdir, f"k_main_{bps}_{mb}.o"),
                      [f"-DRCM_KBPS={bps}", f"-DRCM_KMB={mb}", os.path.join(CSRC, "k_main_inst.cu")]))
     procs = []
     for obj, args in jobs:
@@ -65,11 +72,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise subprocess.CalledProcessError(1, f"nvcc failed for {bad}")
     for obj, _ in procs:
         os.replace(obj + f".tmp{os.getpid()}", obj)
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = lib + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-Xlinker", "--no-undefined", "-o", tmp,
                            *[obj for obj, _ in jobs]])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 CPU_LIB = os.path.join(HERE, "libcpubatch.so")
@@ -91,4 +98,5 @@ def build_cpu(force: bool = False) -> str:
 
 if __name__ == "__main__":
     print(build_cpu(force="--force" in sys.argv))
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    outs = [a[len("--out="):] for a in sys.argv if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, out=outs[0] if outs else None))

@@ -189,7 +189,9 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   p->solo_BS = o.batch_nodes ? std::min(o.batch_nodes, rcm_ksolo_threads()) : rcm_ksolo_threads();
   p->mats_cap = n_max + 1;
   p->gvis_words = n_max / 32 + p->mats_cap + 2;
-  p->spill_cap = n_max;
+  // oversize scratch: children of oversize parents (<= n) + claims bitmaps of
+  // rows longer than the shared-memory bitmap (<= nnz / 64 u64 words)
+  p->spill_cap = n_max + (p->batched_only ? 0 : nnz_max / 64 + 64);
   // ---- multi-block chain path
   if (!p->batched_only) {
     const bool dense = !o.temp_elems && !o.batch_nodes && nnz_max >= 20 * n_max;

@@ -128,6 +128,7 @@ struct ShState {
   int32_t k, written, pos, big_n;
   unsigned long long minkey;
   int64_t spill_base;
+  uint32_t* ovbits;            // oversize claims bitmap (shared memory, or HBM scratch for long rows)
   int32_t big_list[256];
   long long clk[10];           // per-stage cycle accumulators (thread 0)
   long long tclk;

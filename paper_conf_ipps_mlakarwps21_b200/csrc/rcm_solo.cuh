@@ -50,8 +50,10 @@ constexpr int kSoloNT = RCM_SOLO_NT;                // threads per block
 constexpr int kSoloNW = kSoloNT / 32;
 constexpr int kSoloU = RCM_SOLO_U;                  // edge slots per thread per batch
 constexpr int kSoloT = kSoloNT * kSoloU;            // T: edge slots of a batch
-constexpr int kSoloH = 2 * kSoloT;                  // claim-table slots (power of two)
-constexpr int kSoloHBits = __builtin_ctz(kSoloH);
+// claim-table slots: the power of two >= T (a batch has at most T distinct
+// children, so linear probing always finds a free slot; load <= T / H)
+constexpr int kSoloHBits = 32 - __builtin_clz((unsigned)kSoloT - 1u);
+constexpr int kSoloH = 1 << kSoloHBits;
 constexpr int kSoloQ = RCM_SOLO_Q;                  // ring of pending parents (power of two)
 constexpr int kSoloNMax = (1 << 17) - 1;            // shared-memory bitmap capacity (nodes)
 constexpr int kSoloVisW = (kSoloNMax >> 5) + 1;     // bitmap words
@@ -91,15 +93,18 @@ struct SoloArgs {
 constexpr size_t kSoOffVis = 0;
 constexpr size_t kSoOffRing = kSoOffVis + 4 * (size_t)kSoloVisW;
 constexpr size_t kSoOffPar = kSoOffRing + 12 * (size_t)kSoloQ;                 // 5 int arrays of kSoloNT + 1
-constexpr size_t kSoOffLpof = kSoOffPar + 5 * 4 * (size_t)(kSoloNT + 1) + 12;
-constexpr size_t kSoOffCand = (kSoOffLpof + 2 * (size_t)kSoloT + 15) & ~size_t(15);
+constexpr size_t kSoOffLpof = kSoOffPar + 5 * 4 * (size_t)(kSoloNT + 1) + 12;            // u16 per edge slot
+constexpr size_t kSoOffFlp = kSoOffLpof + 2 * (size_t)kSoloT;                            // u16 per thread
+constexpr size_t kSoOffCand = (kSoOffFlp + 2 * (size_t)kSoloNT + 15) & ~size_t(15);
 constexpr size_t kSoOffHash = kSoOffCand + 8 * (size_t)kSoloT;
 constexpr size_t kSoOffRsv = kSoOffHash + 4 * (size_t)kSoloH;                  // big matrices: 8 B entries over hash+rsv
 constexpr size_t kSoloSmem = kSoOffRsv + 4 * (size_t)kSoloH;
-static_assert(kSoloSmem - kSoOffLpof >= 4 * (size_t)kSoloVisW, "GL bitmap overlays lpof..rsv");
+static_assert(kSoloSmem - kSoOffCand >= 4 * (size_t)kSoloVisW, "GL bitmap overlays cand..rsv");
 
 struct SoloSh {
   int32_t wtmp[kSoloNW + 1];
+  int32_t wscan[2][kSoloNW];   // one-barrier scans alternate between the two buffers
+  int32_t nbig[2];             // segments above 16 children, per batch parity
   long long wtmpll[kSoloNW + 1];
   unsigned long long wtmp64[kSoloNW + 1];
   int32_t k, pos, written, rhi, nP, E, cnt, tail, found, big_n;
@@ -137,6 +142,7 @@ __device__ __forceinline__ int32_t* so_p_eo() { return so_p_v() + 2 * (kSoloNT +
 __device__ __forceinline__ int32_t* so_p_cnt() { return so_p_v() + 3 * (kSoloNT + 1); }
 __device__ __forceinline__ int32_t* so_p_pfx() { return so_p_v() + 4 * (kSoloNT + 1); }
 __device__ __forceinline__ uint16_t* so_lpof() { return reinterpret_cast<uint16_t*>(so_base() + kSoOffLpof); }
+__device__ __forceinline__ uint16_t* so_flp() { return reinterpret_cast<uint16_t*>(so_base() + kSoOffFlp); }
 __device__ __forceinline__ unsigned long long* so_cand() {
   return reinterpret_cast<unsigned long long*>(so_base() + kSoOffCand);
 }
@@ -191,6 +197,18 @@ __device__ __forceinline__ unsigned long long so_min_u64(unsigned long long v, S
   return r;
 }
 
+__device__ __forceinline__ unsigned long long so_or_u64(unsigned long long v, SoloSh& sh) {
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) v |= __shfl_xor_sync(0xffffffffu, v, d);
+  if ((threadIdx.x & 31) == 0) sh.wtmp64[threadIdx.x >> 5] = v;
+  __syncthreads();
+  unsigned long long r = 0;
+#pragma unroll
+  for (int w = 0; w < kSoloNW; ++w) r |= sh.wtmp64[w];
+  __syncthreads();
+  return r;
+}
+
 __device__ __forceinline__ bool so_test(const SoloMat& M, int v) {
   const uint32_t w = M.gmem ? __ldcg(M.vis + (v >> 5)) : M.vis[v >> 5];
   return (w >> (v & 31)) & 1u;
@@ -211,9 +229,10 @@ __device__ __forceinline__ void so_zero_bits(uint32_t* bits, int n) {
 __device__ __forceinline__ uint32_t so_hslot(uint32_t c) { return (c * 2654435761u) >> (32 - kSoloHBits); }
 
 // Insert claim (c, e) into the table: per child the minimum edge slot (small
-// matrices: one 32-bit word c:17 | e:15; large: c:32 | e:32).  Returns the slot.
+// matrices: one 32-bit word c:17 | e:15; large: c:32 | e:32).  Returns the
+// slot; *ins = this call created the entry (exactly one claimer per child).
 template <bool kBig>
-__device__ __forceinline__ int so_claim(uint32_t c, uint32_t e) {
+__device__ __forceinline__ int so_claim(uint32_t c, uint32_t e, bool* ins) {
   uint32_t s = so_hslot(c);
   if constexpr (!kBig) {
     volatile uint32_t* h = so_hash();
@@ -222,9 +241,9 @@ __device__ __forceinline__ int so_claim(uint32_t c, uint32_t e) {
       uint32_t cur = h[s];
       if (cur == kEmpty32) {
         cur = atomicCAS(const_cast<uint32_t*>(h) + s, kEmpty32, want);
-        if (cur == kEmpty32) return (int)s;
+        if (cur == kEmpty32) { *ins = true; return (int)s; }
       }
-      if ((cur >> 15) == c) { atomicMin(const_cast<uint32_t*>(h) + s, want); return (int)s; }
+      if ((cur >> 15) == c) { atomicMin(const_cast<uint32_t*>(h) + s, want); *ins = false; return (int)s; }
       s = (s + 1) & (kSoloH - 1);
     }
   } else {
@@ -234,17 +253,32 @@ __device__ __forceinline__ int so_claim(uint32_t c, uint32_t e) {
       unsigned long long cur = h[s];
       if (cur == kKeyMax) {
         cur = atomicCAS(const_cast<unsigned long long*>(h) + s, kKeyMax, want);
-        if (cur == kKeyMax) return (int)s;
+        if (cur == kKeyMax) { *ins = true; return (int)s; }
       }
-      if ((uint32_t)(cur >> 32) == c) { atomicMin(const_cast<unsigned long long*>(h) + s, want); return (int)s; }
+      if ((uint32_t)(cur >> 32) == c) {
+        atomicMin(const_cast<unsigned long long*>(h) + s, want);
+        *ins = false;
+        return (int)s;
+      }
       s = (s + 1) & (kSoloH - 1);
     }
   }
 }
+// Winning (minimum) edge slot of the child in table slot s.
 template <bool kBig>
-__device__ __forceinline__ bool so_won(int s, uint32_t c, uint32_t e) {
-  if constexpr (!kBig) return so_hash()[s] == ((c << 15) | e);
-  else return so_hash64()[s] == (((unsigned long long)c << 32) | e);
+__device__ __forceinline__ int so_winner(int s) {
+  if constexpr (!kBig) return (int)(so_hash()[s] & 0x7fffu);
+  else return (int)(uint32_t)so_hash64()[s];
+}
+// Local parent of edge slot e: the largest lp with p_eo[lp] <= e.
+__device__ __forceinline__ int so_find_lp(int e, int nP) {
+  const int32_t* eo = so_p_eo();
+  int lo = 0, hi = nP - 1;
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (eo[mid] <= e) lo = mid; else hi = mid - 1;
+  }
+  return lo;
 }
 template <bool kBig>
 __device__ __forceinline__ void so_unclaim(int s) {
@@ -270,7 +304,7 @@ static __device__ void so_radix_sort_global(unsigned long long* a, unsigned long
   const unsigned long long first = __ldcg(a);
   unsigned long long diff = 0;
   for (int i = threadIdx.x; i < n; i += kSoloNT) diff |= __ldcg(a + i) ^ first;
-  diff = ~so_min_u64(~diff, sh);                              // block OR
+  diff = so_or_u64(diff, sh);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const unsigned lt = (1u << lane) - 1;
   unsigned long long* src = a;
@@ -415,17 +449,21 @@ static __device__ int so_next_seed(const SoloMat& M, SoloSh& sh) {
   }
 }
 
-// Place a root at position q (thread 0): perm, iperm, placed bit, ring.
-__device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int s, int q) {
-  M.perm[M.n - 1 - q] = s;
-  if (a.iperm) a.iperm[M.node_base + s] = M.n - 1 - q;
-  so_set(M, M.vis, s);
-  if (sh.rhi == q) {   // ring contiguous up to the output end
-    so_ring_v()[q & (kSoloQ - 1)] = s;
-    so_ring_rs()[q & (kSoloQ - 1)] = __ldg(M.rp + s);
-    so_ring_d()[q & (kSoloQ - 1)] = so_deg(M, s);
-    sh.rhi = q + 1;
+// Place a root at position q: perm, iperm, placed bit (thread 0) and the ring
+// entry if the ring is contiguous up to q (rhi == q; every thread updates its
+// copy of rhi).
+__device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& M, int s, int q, int& rhi) {
+  if (threadIdx.x == 0) {
+    M.perm[M.n - 1 - q] = s;
+    if (a.iperm) a.iperm[M.node_base + s] = M.n - 1 - q;
+    so_set(M, M.vis, s);
+    if (rhi == q) {
+      so_ring_v()[q & (kSoloQ - 1)] = s;
+      so_ring_rs()[q & (kSoloQ - 1)] = __ldg(M.rp + s);
+      so_ring_d()[q & (kSoloQ - 1)] = so_deg(M, s);
+    }
   }
+  if (rhi == q) rhi = q + 1;
 }
 
 // ------------------------------------------------------------ validation
@@ -471,111 +509,223 @@ static __device__ bool so_validate(const SoloArgs& a, const SoloMat& M, SoloSh& 
 }
 
 // ---------------------------------------------------------------- batches
-// Sort each parent's winners by (valence, id): <= 16 by one thread, else one warp.
-static __device__ void so_sort_segments(int nP, SoloSh& sh) {
-  if (threadIdx.x == 0) sh.big_n = 0;
-  __syncthreads();
-  unsigned long long* cand = so_cand();
-  for (int lp = threadIdx.x; lp < nP; lp += kSoloNT) {
-    const int n = so_p_cnt()[lp];
-    if (n <= 1) continue;
-    unsigned long long* a = cand + so_p_eo()[lp];
-    if (n <= 16) {
-      for (int i = 1; i < n; ++i) {
-        const unsigned long long x = a[i];
-        int j = i - 1;
-        while (j >= 0 && a[j] > x) { a[j + 1] = a[j]; --j; }
-        a[j + 1] = x;
-      }
-    } else {
-      sh.big_list[atomicAdd(&sh.big_n, 1)] = lp;
-    }
-  }
-  __syncthreads();
-  const int nbig = sh.big_n;
+// Exclusive block scan with ONE barrier: warp totals go to buffer `buf`,
+// consecutive calls alternate buffers (a buffer is rewritten only after every
+// thread has passed the other buffer's barrier).
+__device__ __forceinline__ int so_scan1(int v, int32_t* buf, int& total) {
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  for (int b = wid; b < nbig; b += kSoloNW) {
-    const int lp = sh.big_list[b];
-    bitonic_sort_flip(cand + so_p_eo()[lp], so_p_cnt()[lp], lane, 32, [] { __syncwarp(); });
+  int x = v;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, x, d);
+    if (lane >= d) x += y;
   }
+  if (lane == 31) buf[wid] = x;
+  __syncthreads();
+  int base = 0, tot = 0;
+#pragma unroll
+  for (int w = 0; w < kSoloNW; ++w) {
+    const int t = buf[w];
+    base += w < wid ? t : 0;
+    tot += t;
+  }
+  total = tot;
+  return base + x - v;
+}
+
+// Traversal state, block-uniform, held in registers by every thread.
+struct SoloPos {
+  int pos;      // next parent position of o
+  int written;  // next output position of o
+  int rhi;      // the ring holds positions [pos, rhi) (small matrices; -1: unused)
+  int par;      // batch parity (scan / counter buffers)
+};
+
+// A parent whose valence exceeds T (P:L814-839): its row in chunks of T edge
+// slots, children to HBM scratch, one block radix sort by (valence, id).
+template <bool kBig>
+static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& sh, SoloPos& S, int rs, int D) {
+  unsigned long long* keys = a.spill + M.node_base;
+  if (threadIdx.x == 0) sh.cnt = 0;
+  __syncthreads();
+  for (int c0 = 0; c0 < D; c0 += kSoloT) {
+    int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
+    bool ins[kSoloU];
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      const int e = c0 + threadIdx.x * kSoloU + u;
+      cc[u] = e < D ? __ldg(M.col + rs + e) : -1;
+      ins[u] = false;
+    }
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      if (cc[u] >= 0 && !so_test(M, cc[u])) {
+        slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x * kSoloU + u), &ins[u]);
+        if (ins[u]) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+      }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) {
+      if (ins[u]) {   // one parent: every child is kept, once (duplicates share the entry)
+        const int idx = atomicAdd(&sh.cnt, 1);
+        keys[idx] = ((unsigned long long)(uint32_t)(cre[u] - crs[u]) << 32) | (uint32_t)cc[u];
+        so_set(M, M.vis, cc[u]);
+        so_unclaim<kBig>(slot[u]);
+      }
+    }
+    __syncthreads();
+  }
+  const int C = sh.cnt;
+  if (!(a.flags & F_NO_SORT)) {
+    so_radix_sort_global(keys, a.spill + a.spill_cap + M.node_base, C, sh);
+    so_hash_reset<kBig>();   // the sort's digit counters overlaid the table
+  }
+  const int last = M.n - 1;
+  for (int i = threadIdx.x; i < C; i += kSoloNT) {
+    const int c = (int)(uint32_t)__ldcg(keys + i);
+    M.perm[last - S.written - i] = c;
+    if (a.iperm) a.iperm[M.node_base + c] = last - S.written - i;
+  }
+  if (threadIdx.x == 0) { ++sh.st_exec; ++sh.st_over; }
+  S.pos += 1;
+  S.written += C;   // the ring is not extended: these parents are refilled from perm
   __syncthreads();
 }
 
-// One batch of parents [pos, pos + nP) whose edges fit the T slots.
+// One batch (P:L749-792 on one block): parents [pos, pos + nP) from the ring,
+// the longest prefix (<= B_s) whose valences fit the T edge slots; thread t
+// owns edge slots [U t, U t + U).  The first claimer of a child (exactly one
+// per child) loads its row_ptr and files it under the winning (minimum edge
+// slot = earliest) parent; thread lp sorts parent lp's children and writes
+// them out.  Six block barriers per batch.
 template <bool kBig>
-static __device__ void so_batch(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int nP) {
-  const int E = so_p_eo()[nP];
-  const int pos = sh.pos, written = sh.written;
-  // edge slot -> local parent, one warp per parent
-  {
-    const int lane = threadIdx.x & 31;
-    for (int lp = threadIdx.x >> 5; lp < nP; lp += kSoloNW) {
-      const int eb = so_p_eo()[lp], ee = so_p_eo()[lp + 1];
-      for (int j = eb + lane; j < ee; j += 32) so_lpof()[j] = (uint16_t)lp;
+static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, SoloPos& S) {
+  const int last = M.n - 1;
+  const int t = threadIdx.x;
+  // ---- refill the ring from perm when it runs low
+  int rhi = S.rhi;
+  if (kBig || (rhi < S.written && rhi - S.pos < a.BS)) {
+    const int lo = kBig ? S.pos : rhi;
+    const int hi = min(S.written, S.pos + kSoloQ);
+    for (int q = lo + t; q < hi; q += kSoloNT) {
+      const int v = __ldcg(M.perm + last - q);
+      const int r0 = __ldg(M.rp + v);
+      so_ring_v()[q & (kSoloQ - 1)] = v;
+      so_ring_rs()[q & (kSoloQ - 1)] = r0;
+      so_ring_d()[q & (kSoloQ - 1)] = __ldg(M.rp + v + 1) - r0;
     }
+    rhi = hi;
+    if (!kBig) S.rhi = hi;
+    __syncthreads();
   }
-  __syncthreads();
-  // discover: columns, placed test, claims; child row_ptr loads in flight
+  // ---- parents
+  const int pos = S.pos, written = S.written;
+  const int avail = min(a.BS, rhi - pos);
+  const int d = t < avail ? so_ring_d()[(pos + t) & (kSoloQ - 1)] : 0;
+  int E;
+  const int eo = so_scan1(d, sh.wscan[0], E);
+  const bool fit = t < avail && eo + d <= kSoloT;
+  if (fit) {
+    so_p_v()[t] = so_ring_v()[(pos + t) & (kSoloQ - 1)];
+    so_p_rs()[t] = so_ring_rs()[(pos + t) & (kSoloQ - 1)];
+    so_p_eo()[t] = eo;
+    so_p_eo()[t + 1] = eo + d;   // == the next parent's offset; the last one ends the slots
+    so_p_cnt()[t] = 0;
+    // owner of the first slot of every U-slot group this parent covers
+    for (int g = (eo + kSoloU - 1) / kSoloU; g * kSoloU < eo + d; ++g) so_flp()[g] = (uint16_t)t;
+  }
+  const int nP = __syncthreads_count(fit);
+  if (nP == 0) {   // the first parent alone exceeds T
+    so_oversize<kBig>(a, M, sh, S, so_ring_rs()[pos & (kSoloQ - 1)], so_ring_d()[pos & (kSoloQ - 1)]);
+    return;
+  }
+  E = so_p_eo()[nP];
+  if (t == 0 && a.collect_stats) {   // does this batch combine the outputs of several earlier batches?
+    while (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] <= pos) ++sh.grp_h;
+    if (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] < pos + nP) ++sh.st_comb;
+  }
+  // ---- discover: columns, placed test, claims; first claimers load the child's row_ptr
+  const int e0 = t * kSoloU;
   int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
+  bool ins[kSoloU];
+  {
+    int lp = e0 < E ? so_flp()[t] : 0;
 #pragma unroll
-  for (int u = 0; u < kSoloU; ++u) {
-    const int e = threadIdx.x + u * kSoloNT;
-    cc[u] = -1;
-    if (e < E) {
-      const int lp = so_lpof()[e];
-      cc[u] = __ldg(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
+    for (int u = 0; u < kSoloU; ++u) {
+      const int e = e0 + u;
+      cc[u] = -1;
+      ins[u] = false;
+      if (e < E) {
+        while (so_p_eo()[lp + 1] <= e) ++lp;
+        so_lpof()[e] = (uint16_t)lp;
+        cc[u] = __ldg(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
+      }
     }
   }
 #pragma unroll
   for (int u = 0; u < kSoloU; ++u) {
-    if (cc[u] >= 0 && so_test(M, cc[u])) cc[u] = -1;   // placed (self-loops included)
-    if (cc[u] >= 0) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+    if (cc[u] >= 0 && !so_test(M, cc[u])) {   // placed nodes (self-loops included) are skipped
+      slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(e0 + u), &ins[u]);
+      if (ins[u]) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+    }
   }
-#pragma unroll
-  for (int u = 0; u < kSoloU; ++u)
-    if (cc[u] >= 0) slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT));
   __syncthreads();
-  // winners: the minimum edge slot per child = the earliest parent
+  // ---- file every child under the minimum edge slot's parent
   int won = 0;
 #pragma unroll
   for (int u = 0; u < kSoloU; ++u) {
-    const int e = threadIdx.x + u * kSoloNT;
-    if (cc[u] >= 0 && so_won<kBig>(slot[u], (uint32_t)cc[u], (uint32_t)e)) {
-      const int lp = so_lpof()[e];
+    if (ins[u]) {
+      const int lp = so_lpof()[so_winner<kBig>(slot[u])];
       const int idx = atomicAdd(&so_p_cnt()[lp], 1);
-      const unsigned long long d = (unsigned long long)(uint32_t)(cre[u] - crs[u]);
+      const unsigned long long dg = (unsigned long long)(uint32_t)(cre[u] - crs[u]);
       unsigned long long key;
       if constexpr (!kBig) {
         so_rsv()[slot[u]] = crs[u];
-        key = (d << 32) | ((unsigned long long)(uint32_t)cc[u] << 15) | (uint32_t)slot[u];
+        key = (dg << 32) | ((unsigned long long)(uint32_t)cc[u] << 15) | (uint32_t)slot[u];
       } else {
-        key = (d << 32) | (uint32_t)cc[u];
+        key = (dg << 32) | (uint32_t)cc[u];
       }
       so_cand()[so_p_eo()[lp] + idx] = key;
       so_set(M, M.vis, cc[u]);
+      so_unclaim<kBig>(slot[u]);   // each entry is read by its creator only
       ++won;
     }
   }
   __syncthreads();
-#pragma unroll
-  for (int u = 0; u < kSoloU; ++u)
-    if (cc[u] >= 0) so_unclaim<kBig>(slot[u]);   // (table reads are done)
-  if (!(a.flags & F_NO_SORT)) so_sort_segments(nP, sh);
-  // output positions: exclusive prefix of the per-parent counts
+  // ---- thread lp: sort parent lp's children by (valence, id) (C-1)
+  const int par = S.par;
+  const int mycnt = t < nP ? so_p_cnt()[t] : 0;
+  unsigned long long* seg = so_cand() + (t < nP ? so_p_eo()[t] : 0);
+  if (mycnt > 1 && !(a.flags & F_NO_SORT)) {
+    if (mycnt <= 16) {
+      for (int i = 1; i < mycnt; ++i) {
+        const unsigned long long x = seg[i];
+        int j = i - 1;
+        while (j >= 0 && seg[j] > x) { seg[j + 1] = seg[j]; --j; }
+        seg[j + 1] = x;
+      }
+    } else {
+      sh.big_list[atomicAdd(&sh.nbig[par], 1)] = t;
+    }
+  }
+  // ---- output positions: exclusive prefix of the per-parent counts
   int tot;
-  const int mycnt = threadIdx.x < nP ? so_p_cnt()[threadIdx.x] : 0;
-  const int pf = so_scan<int32_t>(mycnt, sh.wtmp, tot);
-  if (threadIdx.x < nP) so_p_pfx()[threadIdx.x] = pf;
-  __syncthreads();
+  const int pf = so_scan1(mycnt, sh.wscan[1], tot);
+  const int nbig = sh.nbig[par];
+  if (nbig) {   // segments above 16 children: one warp each
+    const int lane = t & 31, wid = t >> 5;
+    for (int b = wid; b < nbig; b += kSoloNW) {
+      const int lp = sh.big_list[b];
+      bitonic_sort_flip(so_cand() + so_p_eo()[lp], so_p_cnt()[lp], lane, 32, [] { __syncwarp(); });
+    }
+    __syncthreads();
+  }
   const int pos_new = pos + nP;
-  const bool ring_ok = !kBig && sh.rhi == written;
-  const int last = M.n - 1;
-  for (int i = threadIdx.x; i < E; i += kSoloNT) {
-    const int lp = so_lpof()[i];
-    const int j = i - so_p_eo()[lp];
-    if (j >= so_p_cnt()[lp]) continue;
-    const unsigned long long key = so_cand()[i];
-    const int q = written + so_p_pfx()[lp] + j;
+  const bool ring_ok = !kBig && S.rhi == written;
+  for (int j = 0; j < mycnt; ++j) {
+    const unsigned long long key = seg[j];
+    const int q = written + pf + j;
     int c;
     if constexpr (!kBig) c = (int)((key >> 15) & 0x1ffffu);
     else c = (int)(uint32_t)key;
@@ -590,147 +740,46 @@ static __device__ void so_batch(const SoloArgs& a, const SoloMat& M, SoloSh& sh,
     }
   }
   if (a.collect_stats && won) atomicAdd(reinterpret_cast<unsigned long long*>(&sh.st_claim), (unsigned long long)won);
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    sh.pos = pos_new;
-    sh.written = written + tot;
-    if (ring_ok) sh.rhi = min(written + tot, pos_new + kSoloQ);
+  if (t == 0) {
+    sh.nbig[par ^ 1] = 0;   // the next batch's counter (this one is read above)
     ++sh.st_exec;
     if (a.collect_stats && tot > 0 && sh.grp_t - sh.grp_h < kSoloGrp) sh.grp[(sh.grp_t++) & (kSoloGrp - 1)] = written;
   }
+  S.pos = pos_new;
+  S.written = written + tot;
+  if (ring_ok) S.rhi = min(written + tot, pos_new + kSoloQ);
+  S.par = par ^ 1;
   __syncthreads();
-}
-
-// A parent whose valence exceeds T (P:L814-839): its row in chunks of T edge
-// slots, winners to HBM scratch, one block radix sort by (valence, id).
-template <bool kBig>
-static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int rs, int D) {
-  unsigned long long* keys = a.spill + M.node_base;
-  if (threadIdx.x == 0) sh.cnt = 0;
-  __syncthreads();
-  for (int c0 = 0; c0 < D; c0 += kSoloT) {
-    int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
-#pragma unroll
-    for (int u = 0; u < kSoloU; ++u) {
-      const int e = c0 + threadIdx.x + u * kSoloNT;
-      cc[u] = e < D ? __ldg(M.col + rs + e) : -1;
-    }
-#pragma unroll
-    for (int u = 0; u < kSoloU; ++u) {
-      if (cc[u] >= 0 && so_test(M, cc[u])) cc[u] = -1;
-      if (cc[u] >= 0) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
-    }
-#pragma unroll
-    for (int u = 0; u < kSoloU; ++u)
-      if (cc[u] >= 0) slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT));
-    __syncthreads();
-#pragma unroll
-    for (int u = 0; u < kSoloU; ++u) {
-      if (cc[u] >= 0 && so_won<kBig>(slot[u], (uint32_t)cc[u], (uint32_t)(threadIdx.x + u * kSoloNT))) {
-        const int idx = atomicAdd(&sh.cnt, 1);
-        keys[idx] = ((unsigned long long)(uint32_t)(cre[u] - crs[u]) << 32) | (uint32_t)cc[u];
-        so_set(M, M.vis, cc[u]);
-      }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int u = 0; u < kSoloU; ++u)
-      if (cc[u] >= 0) so_unclaim<kBig>(slot[u]);
-    __syncthreads();
-  }
-  const int C = sh.cnt;
-  if (!(a.flags & F_NO_SORT)) {
-    so_radix_sort_global(keys, a.spill + a.spill_cap + M.node_base, C, sh);
-    so_hash_reset<kBig>();   // the sort's digit counters overlaid the table
-  }
-  const int written = sh.written, last = M.n - 1;
-  for (int i = threadIdx.x; i < C; i += kSoloNT) {
-    const int c = (int)(uint32_t)__ldcg(keys + i);
-    M.perm[last - written - i] = c;
-    if (a.iperm) a.iperm[M.node_base + c] = last - written - i;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    sh.pos += 1;
-    sh.written = written + C;   // the ring is not extended: these parents are refilled from perm
-    ++sh.st_exec;
-    ++sh.st_over;
-  }
-  __syncthreads();
-}
-
-// Choose the next batch: refill the ring from perm when it runs low, then the
-// longest prefix of [pos, rhi) (at most B_s) whose valences fit T.
-template <bool kBig>
-static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh) {
-  const int pos = sh.pos, written = sh.written;
-  int rhi = sh.rhi;
-  const int last = M.n - 1;
-  if (kBig || (rhi < written && rhi - pos < a.BS)) {
-    const int lo = kBig ? pos : max(rhi, pos);
-    const int hi = min(written, pos + kSoloQ);
-    for (int q = lo + threadIdx.x; q < hi; q += kSoloNT) {
-      const int v = __ldcg(M.perm + last - q);
-      const int r0 = __ldg(M.rp + v);
-      so_ring_v()[q & (kSoloQ - 1)] = v;
-      so_ring_rs()[q & (kSoloQ - 1)] = r0;
-      so_ring_d()[q & (kSoloQ - 1)] = __ldg(M.rp + v + 1) - r0;
-    }
-    rhi = hi;
-    __syncthreads();
-    if (threadIdx.x == 0 && !kBig) sh.rhi = hi;   // big matrices: the ring is only a staging buffer
-  }
-  const int avail = min(a.BS, rhi - pos);
-  const int t = threadIdx.x;
-  const int d = t < avail ? so_ring_d()[(pos + t) & (kSoloQ - 1)] : 0;
-  int tot;
-  const int eo = so_scan<int32_t>(d, sh.wtmp, tot);
-  const bool fit = t < avail && eo + d <= kSoloT;
-  if (fit) {
-    so_p_v()[t] = so_ring_v()[(pos + t) & (kSoloQ - 1)];
-    so_p_rs()[t] = so_ring_rs()[(pos + t) & (kSoloQ - 1)];
-    so_p_eo()[t] = eo;
-    so_p_cnt()[t] = 0;
-  }
-  const int nP = __syncthreads_count(fit);
-  if (nP == 0) {   // the first parent alone exceeds T
-    so_oversize<kBig>(a, M, sh, so_ring_rs()[pos & (kSoloQ - 1)], so_ring_d()[pos & (kSoloQ - 1)]);
-    return;
-  }
-  if (t == nP - 1) so_p_eo()[nP] = eo + d;
-  if (t == 0 && a.collect_stats) {   // does this batch combine several earlier outputs?
-    while (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] <= pos) ++sh.grp_h;
-    if (sh.grp_h < sh.grp_t && sh.grp[sh.grp_h & (kSoloGrp - 1)] < pos + nP) ++sh.st_comb;
-  }
-  __syncthreads();
-  so_batch<kBig>(a, M, sh, nP);
 }
 
 template <bool kBig>
 static __device__ void so_traverse(const SoloArgs& a, const SoloMat& M, SoloSh& sh, int seed) {
+  SoloPos S;
+  S.pos = 0;
+  S.written = 0;
+  S.rhi = kBig ? -1 : 0;
+  S.par = 0;
   if (threadIdx.x == 0) {
-    sh.pos = 0; sh.written = 0; sh.rhi = kBig ? -1 : 0;
     sh.grp_h = sh.grp_t = 0;
-    so_place_root(a, M, sh, seed, 0);
-    sh.written = 1;
+    sh.nbig[0] = sh.nbig[1] = 0;
     ++sh.st_comp;
   }
+  so_place_root(a, M, seed, 0, S.rhi);
+  S.written = 1;
   __syncthreads();
   for (;;) {
-    if (sh.pos == sh.written) {   // component exhausted (C-6)
-      if (sh.written >= M.n) break;
+    if (S.pos == S.written) {   // component exhausted (C-6)
+      if (S.written >= M.n) break;
       int s = so_next_seed(M, sh);
       if (s < 0) { if (threadIdx.x == 0) atomicCAS(&a.ctl->status, 0, ST_BAD_CSR); break; }
-      if (a.mode == RCM_START_PSEUDO_PERIPHERAL) s = so_gl(M, sh.written, s, sh);
-      if (threadIdx.x == 0) {
-        so_place_root(a, M, sh, s, sh.written);
-        sh.written += 1;
-        ++sh.st_comp;
-      }
+      if (a.mode == RCM_START_PSEUDO_PERIPHERAL) s = so_gl(M, S.written, s, sh);
+      so_place_root(a, M, s, S.written, S.rhi);
+      S.written += 1;
+      if (threadIdx.x == 0) ++sh.st_comp;
       __syncthreads();
       continue;
     }
-    so_step<kBig>(a, M, sh);
+    so_step<kBig>(a, M, sh, S);
   }
 }
 
@@ -760,7 +809,7 @@ static __device__ void so_matrix(const SoloArgs& a, int k, SoloSh& sh) {
     M.bvis = a.gvis + a.gvis_words + w;
   } else {
     M.vis = reinterpret_cast<uint32_t*>(so_base() + kSoOffVis);
-    M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffLpof);   // overlays the batch scratch
+    M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffCand);   // overlays the batch scratch
   }
   if (a.validate && !so_validate(a, M, sh)) return;
   int seed;

@@ -154,14 +154,20 @@ static __device__ void block_radix_sort_global(unsigned long long* a, unsigned l
 // (valence, id) there, written out, and cut into batches chunk by chunk.
 static __device__ bool oversize_discover(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                   ShState& sh, uint32_t key, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
   const int nw = (D + 31) >> 5;
-  if (nw > 2 * (kp.T + 1)) {
-    if (threadIdx.x == 0) latch_error(kp.ctl, ST_CAPACITY);
-    __syncthreads();
-    return false;
+  if (threadIdx.x == 0) {
+    sh.ovbits = reinterpret_cast<uint32_t*>(sm_cand(kp));
+    if (nw > 2 * (kp.T + 1)) {   // row longer than the shared-memory bitmap: HBM scratch
+      const long long base = atomicAdd(&kp.ctl->spill_cursor, (nw + 1) >> 1);
+      if (base + ((nw + 1) >> 1) > kp.spill_cap) { latch_error(kp.ctl, ST_CAPACITY); sh.ovbits = nullptr; }
+      else sh.ovbits = reinterpret_cast<uint32_t*>(kp.spill + base);
+    }
   }
+  __syncthreads();
+  uint32_t* bits = sh.ovbits;
+  if (!bits) return false;
   for (int i = threadIdx.x; i < nw; i += kThreads) bits[i] = 0;
+  __threadfence_block();
   __syncthreads();
   unsigned long long* word = kp.word + P.node_base;
   const int32_t* col = kp.col_idx + P.ci_base + rs;
@@ -178,21 +184,27 @@ static __device__ bool oversize_discover(const KParams& kp, const Problem& P, co
     int tot = block_reduce_sum<int32_t>(claims, sh.wtmp32);
     if (threadIdx.x == 0) stat_add(kp, &kp.stats->cand_spec, tot);
   }
+  __threadfence_block();
   __syncthreads();
   return true;
+}
+
+// bitmap word i (shared memory, or HBM written by atomics: read through L2)
+__device__ __forceinline__ uint32_t ov_word(const KParams& kp, const uint32_t* bits, int i) {
+  return __isShared(bits) ? bits[i] : __ldcg(bits + i);
 }
 
 // Rediscover (keep iff owner == key), then count and clamped valence sum.
 static __device__ void oversize_rediscover_count(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                           ShState& sh, uint32_t key, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
+  uint32_t* bits = sh.ovbits;
   const int nw = (D + 31) >> 5;
   const unsigned long long* word = kp.word + P.node_base;
   const int32_t* col = kp.col_idx + P.ci_base + rs;
   int cnt = 0, removed = 0;
   long long val = 0;
   for (int i = threadIdx.x; i < nw; i += kThreads) {
-    uint32_t b = bits[i], keep = b;
+    uint32_t b = ov_word(kp, bits, i), keep = b;
     while (b) {
       int j = __ffs(b) - 1;
       b &= b - 1;
@@ -203,6 +215,7 @@ static __device__ void oversize_rediscover_count(const KParams& kp, const Proble
     }
     bits[i] = keep;
   }
+  __threadfence_block();
   int C = block_reduce_sum<int32_t>(cnt, sh.wtmp32);
   long long V = block_reduce_sum<long long>(val, sh.wtmpll);
   int R = block_reduce_sum<int32_t>(removed, sh.wtmp32);
@@ -217,7 +230,7 @@ static __device__ void oversize_rediscover_count(const KParams& kp, const Proble
 // Gather kept children into spill, sort them.  Returns false on capacity error.
 static __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P, const SmemPtrs& sm,
                                      ShState& sh, int rs, int D) {
-  uint32_t* bits = reinterpret_cast<uint32_t*>(sm_cand(kp));
+  const uint32_t* bits = sh.ovbits;
   const int nw = (D + 31) >> 5;
   const int C = sh.count;
   if (threadIdx.x == 0) {
@@ -234,11 +247,11 @@ static __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P,
   const int per = (nw + kThreads - 1) / kThreads;
   const int b = threadIdx.x * per, e = min(nw, b + per);
   int mine = 0;
-  for (int i = b; i < e; ++i) mine += __popc(bits[i]);
+  for (int i = b; i < e; ++i) mine += __popc(ov_word(kp, bits, i));
   int tot;
   int run = block_exclusive_scan<int32_t>(mine, sh.wtmp32, tot);
   for (int i = b; i < e; ++i) {
-    uint32_t x = bits[i];
+    uint32_t x = ov_word(kp, bits, i);
     while (x) {
       int j = __ffs(x) - 1;
       x &= x - 1;
