@@ -175,6 +175,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
+  if (const char* g = std::getenv("RCM_L2_FETCH")) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, std::atoi(g));
   // ---- batched / small-graph path: many blocks per SM, shared-memory bitmap
   p->solo_smem = rcm_ksolo_smem();
   if (cudaFuncSetAttribute(rcm_ksolo_ptr(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->solo_smem) !=

@@ -98,7 +98,8 @@ constexpr size_t kSoOffFlp = kSoOffLpof + 2 * (size_t)kSoloT;                   
 constexpr size_t kSoOffCand = (kSoOffFlp + 2 * (size_t)kSoloNT + 15) & ~size_t(15);
 constexpr size_t kSoOffHash = kSoOffCand + 8 * (size_t)kSoloT;
 constexpr size_t kSoOffRsv = kSoOffHash + 4 * (size_t)kSoloH;                  // big matrices: 8 B entries over hash+rsv
-constexpr size_t kSoloSmem = kSoOffRsv + 4 * (size_t)kSoloH;
+constexpr size_t kSoOffRdeg = kSoOffRsv + 4 * (size_t)kSoloH;                 // valence per table slot
+constexpr size_t kSoloSmem = kSoOffRdeg + 4 * (size_t)kSoloH;
 static_assert(kSoloSmem - kSoOffCand >= 4 * (size_t)kSoloVisW, "GL bitmap overlays cand..rsv");
 
 struct SoloSh {
@@ -151,6 +152,7 @@ __device__ __forceinline__ unsigned long long* so_hash64() {
   return reinterpret_cast<unsigned long long*>(so_base() + kSoOffHash);
 }
 __device__ __forceinline__ int32_t* so_rsv() { return reinterpret_cast<int32_t*>(so_base() + kSoOffRsv); }
+__device__ __forceinline__ int32_t* so_rdeg() { return reinterpret_cast<int32_t*>(so_base() + kSoOffRdeg); }
 
 // ------------------------------------------------------------- block helpers
 template <typename T>
@@ -212,6 +214,16 @@ __device__ __forceinline__ unsigned long long so_or_u64(unsigned long long v, So
 __device__ __forceinline__ bool so_test(const SoloMat& M, int v) {
   const uint32_t w = M.gmem ? __ldcg(M.vis + (v >> 5)) : M.vis[v >> 5];
   return (w >> (v & 31)) & 1u;
+}
+template <bool kBig>
+__device__ __forceinline__ bool so_placed(const SoloMat& M, int v) {
+  uint32_t w;
+  if constexpr (kBig) w = __ldcg(M.vis + (v >> 5));
+  else w = reinterpret_cast<const uint32_t*>(so_base() + kSoOffVis)[v >> 5];
+  return (w >> (v & 31)) & 1u;
+}
+__device__ __forceinline__ void so_prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 __device__ __forceinline__ void so_set(const SoloMat& M, uint32_t* bits, int v) {
   atomicOr(bits + (v >> 5), 1u << (v & 31));
@@ -559,7 +571,7 @@ static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& 
     }
 #pragma unroll
     for (int u = 0; u < kSoloU; ++u) {
-      if (cc[u] >= 0 && !so_test(M, cc[u])) {
+      if (cc[u] >= 0 && !so_placed<kBig>(M, cc[u])) {
         slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x * kSoloU + u), &ins[u]);
         if (ins[u]) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
       }
@@ -647,15 +659,13 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   }
   // ---- discover: columns, placed test, claims; first claimers load the child's row_ptr
   const int e0 = t * kSoloU;
-  int cc[kSoloU], slot[kSoloU], crs[kSoloU], cre[kSoloU];
-  bool ins[kSoloU];
+  int cc[kSoloU], slot[kSoloU];   // slot >= 0: this thread created the child's table entry
   {
     int lp = e0 < E ? so_flp()[t] : 0;
 #pragma unroll
     for (int u = 0; u < kSoloU; ++u) {
       const int e = e0 + u;
       cc[u] = -1;
-      ins[u] = false;
       if (e < E) {
         while (so_p_eo()[lp + 1] <= e) ++lp;
         so_lpof()[e] = (uint16_t)lp;
@@ -665,9 +675,16 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   }
 #pragma unroll
   for (int u = 0; u < kSoloU; ++u) {
-    if (cc[u] >= 0 && !so_test(M, cc[u])) {   // placed nodes (self-loops included) are skipped
-      slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(e0 + u), &ins[u]);
-      if (ins[u]) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+    slot[u] = -1;
+    if (cc[u] >= 0 && !so_placed<kBig>(M, cc[u])) {   // placed nodes (self-loops included) are skipped
+      bool ins;
+      const int sl = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(e0 + u), &ins);
+      if (ins) {
+        const int r0 = __ldg(M.rp + cc[u]);
+        if constexpr (!kBig) so_rsv()[sl] = r0;   // (big matrices: the 8 B entries overlay rsv)
+        so_rdeg()[sl] = __ldg(M.rp + cc[u] + 1) - r0;
+        slot[u] = sl;
+      }
     }
   }
   __syncthreads();
@@ -675,20 +692,20 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   int won = 0;
 #pragma unroll
   for (int u = 0; u < kSoloU; ++u) {
-    if (ins[u]) {
-      const int lp = so_lpof()[so_winner<kBig>(slot[u])];
+    const int sl = slot[u];
+    if (sl >= 0) {
+      int c, ew;
+      if constexpr (!kBig) { const uint32_t h = so_hash()[sl]; c = (int)(h >> 15); ew = (int)(h & 0x7fffu); }
+      else { const unsigned long long h = so_hash64()[sl]; c = (int)(h >> 32); ew = (int)(uint32_t)h; }
+      const int lp = so_lpof()[ew];
       const int idx = atomicAdd(&so_p_cnt()[lp], 1);
-      const unsigned long long dg = (unsigned long long)(uint32_t)(cre[u] - crs[u]);
+      const unsigned long long dg = (unsigned long long)(uint32_t)so_rdeg()[sl];
       unsigned long long key;
-      if constexpr (!kBig) {
-        so_rsv()[slot[u]] = crs[u];
-        key = (dg << 32) | ((unsigned long long)(uint32_t)cc[u] << 15) | (uint32_t)slot[u];
-      } else {
-        key = (dg << 32) | (uint32_t)cc[u];
-      }
+      if constexpr (!kBig) key = (dg << 32) | ((unsigned long long)(uint32_t)c << 15) | (uint32_t)sl;
+      else key = (dg << 32) | (uint32_t)c;
       so_cand()[so_p_eo()[lp] + idx] = key;
-      so_set(M, M.vis, cc[u]);
-      so_unclaim<kBig>(slot[u]);   // each entry is read by its creator only
+      so_set(M, M.vis, c);
+      so_unclaim<kBig>(sl);   // each entry is read by its creator only
       ++won;
     }
   }
