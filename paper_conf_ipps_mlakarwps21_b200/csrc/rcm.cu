@@ -42,6 +42,7 @@ struct rcm_plan {
   int64_t mats_cap = 0, gvis_words = 0;
   int32_t* order = nullptr;
   uint32_t* gvis = nullptr;
+  int2* pend = nullptr;
   int solo_BS = 256;
   bool batched_only = false;
 };
@@ -76,7 +77,7 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->pend, p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
                   p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
@@ -123,6 +124,7 @@ static rcm_status_t plan_alloc(rcm_plan* p) {
   // batched / small-graph path (rcm_solo.cuh)
   AL(p->order, 4 * p->mats_cap);
   AL(p->gvis, 4 * 2 * p->gvis_words);
+  AL(p->pend, 8 * n);
   if (!p->batched_only) {   // multi-block chain + components + GL finder
     const int64_t tiles = (n + kSortTile - 1) / kSortTile + 1;
     AL(p->word, 8 * n);
@@ -175,7 +177,6 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   int smem_optin = 0, smem_sm = 0;
   cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, p->device);
   cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, p->device);
-  if (const char* g = std::getenv("RCM_L2_FETCH")) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, std::atoi(g));
   // ---- batched / small-graph path: many blocks per SM, shared-memory bitmap
   p->solo_smem = rcm_ksolo_smem();
   if (cudaFuncSetAttribute(rcm_ksolo_ptr(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->solo_smem) !=
@@ -189,7 +190,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   p->solo_blocks = occ_s * p->num_sms;
   p->solo_BS = o.batch_nodes ? std::min(o.batch_nodes, rcm_ksolo_threads()) : rcm_ksolo_threads();
   p->mats_cap = n_max + 1;
-  p->gvis_words = n_max / 32 + p->mats_cap + 2;
+  p->gvis_words = n_max / 32 + 2;   // bitmaps packed over all nodes (one bit each)
   // oversize scratch: children of oversize parents (<= n) + claims bitmaps of
   // rows longer than the shared-memory bitmap (<= nnz / 64 u64 words)
   p->spill_cap = n_max + (p->batched_only ? 0 : nnz_max / 64 + 64);
@@ -314,6 +315,7 @@ static rcm_status_t launch_solo(rcm_plan* p, SoloArgs& sa, cudaStream_t s) {
   sa.gvis_words = p->gvis_words;
   sa.spill = p->spill;
   sa.spill_cap = p->spill_cap;
+  sa.pend = p->pend;
   sa.ctl = p->ctl;
   sa.stats = p->stats;
   sa.validate = p->opt.validate;

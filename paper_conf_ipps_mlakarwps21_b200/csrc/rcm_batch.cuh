@@ -261,7 +261,9 @@ static __device__ void discover(const KParams& kp, const Problem& P, const SmemP
   // before any result is used: the three dependent round trips (column,
   // owner word, atomicMin) are paid once per round instead of once per edge.
   for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
-    int c[kDiscU], lps[kDiscU];
+    // the local parent of a slot is re-read from shared memory (lpof) where it
+    // is needed instead of being held in registers across the three steps
+    int c[kDiscU];
     unsigned long long w[kDiscU];
 #pragma unroll
     for (int u = 0; u < kDiscU; ++u) {
@@ -269,7 +271,6 @@ static __device__ void discover(const KParams& kp, const Problem& P, const SmemP
       c[u] = -1;
       if (e < E) {
         const int lp = sm_lpof(kp)[e];
-        lps[u] = lp;
         c[u] = __ldg(col + sm_p_rs(kp)[lp] + (e - sm_p_eo(kp)[lp]));
       }
     }
@@ -277,18 +278,21 @@ static __device__ void discover(const KParams& kp, const Problem& P, const SmemP
     for (int u = 0; u < kDiscU; ++u) w[u] = c[u] >= 0 ? ld_weak_u64(word + c[u]) : 0ull;   // prefilter
 #pragma unroll
     for (int u = 0; u < kDiscU; ++u) {
-      const uint32_t key = kfirst + (uint32_t)lps[u];
-      if (c[u] >= 0 && (uint32_t)(w[u] >> 32) > key)
+      if (c[u] < 0) continue;
+      const uint32_t key = kfirst + (uint32_t)sm_lpof(kp)[e0 + u * kThreads];
+      if ((uint32_t)(w[u] >> 32) > key)
         w[u] = atomicMin(word + c[u], ((unsigned long long)key << 32) | (w[u] & 0xffffffffull));
       else
         c[u] = -1;
     }
 #pragma unroll
     for (int u = 0; u < kDiscU; ++u) {
-      const uint32_t key = kfirst + (uint32_t)lps[u];
+      if (c[u] < 0) continue;
+      const int lp = sm_lpof(kp)[e0 + u * kThreads];
+      const uint32_t key = kfirst + (uint32_t)lp;
       const uint32_t ow = (uint32_t)(w[u] >> 32);
-      if (c[u] >= 0 && ow > key) {
-        int slot = sm_p_eo(kp)[lps[u]] + atomicAdd(&sm_p_cnt(kp)[lps[u]], 1);
+      if (ow > key) {
+        int slot = sm_p_eo(kp)[lp] + atomicAdd(&sm_p_cnt(kp)[lp], 1);
         sm_cand(kp)[slot] = ((w[u] & 0xffffffffull) << 32) | (uint32_t)c[u];
         steal |= (ow <= klast);   // taken from a sibling parent of this batch
         ++claims;

@@ -402,6 +402,10 @@ static __device__ __noinline__ void chain_worker_mb(const KParams& kp, const Pro
       if (threadIdx.x == 0) rcm_ctx_base = c ? cbytes : 0u;
       __syncthreads();
       const int ph = s.mb;
+      // every thread has read the phase before thread 0 may overwrite it below
+      // (compute-sanitizer racecheck: a late reader could otherwise follow the
+      // new phase into a different sequence of block barriers)
+      __syncthreads();
       int nx = ph;
       if (ph == PH_IDLE) {
         if (threadIdx.x == 0) {

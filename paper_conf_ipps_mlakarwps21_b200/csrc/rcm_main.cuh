@@ -70,15 +70,24 @@ static __device__ void prologue_phase(const KParams& kp, const MainArgs& a, ShSt
 }
 
 // validate == 2: structural symmetry -- for every (u, c) the row of c holds u.
+// Binary search (sorted rows: O(nnz log deg)), linear scan only when the
+// search misses (unsorted rows).
 static __device__ void validate_sym_phase(const KParams& kp, int n) {
   int bad = 0;
   for (int u = gtid(); u < n; u += gthreads(kp)) {
     for (int e = __ldg(kp.row_ptr + u); e < __ldg(kp.row_ptr + u + 1); ++e) {
       const int c = __ldg(kp.col_idx + e);
       if (c < 0 || c >= n) { bad = 1; continue; }
+      const int b0 = __ldg(kp.row_ptr + c), b1 = __ldg(kp.row_ptr + c + 1) - 1;
+      int lo = b0, hi = b1;
       bool found = false;
-      for (int f = __ldg(kp.row_ptr + c); f < __ldg(kp.row_ptr + c + 1) && !found; ++f)
-        found = __ldg(kp.col_idx + f) == u;
+      while (lo <= hi) {
+        const int mid = (lo + hi) >> 1;
+        const int x = __ldg(kp.col_idx + mid);
+        if (x == u) { found = true; break; }
+        if (x < u) lo = mid + 1; else hi = mid - 1;
+      }
+      for (int f = b0; f <= b1 && !found; ++f) found = __ldg(kp.col_idx + f) == u;
       bad |= !found;
     }
   }

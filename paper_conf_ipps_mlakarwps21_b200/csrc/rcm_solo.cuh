@@ -46,6 +46,10 @@ namespace rcm {
 #ifndef RCM_SOLO_Q
 #define RCM_SOLO_Q 512
 #endif
+#ifndef RCM_SOLO_PEND
+#define RCM_SOLO_PEND 1
+#endif
+constexpr bool kSoloPend = RCM_SOLO_PEND != 0;     // ring overflow kept as (row start, valence)
 constexpr int kSoloNT = RCM_SOLO_NT;                // threads per block
 constexpr int kSoloNW = kSoloNT / 32;
 constexpr int kSoloU = RCM_SOLO_U;                  // edge slots per thread per batch
@@ -75,6 +79,9 @@ struct SoloArgs {
   uint32_t* gvis;             // HBM bitmaps for matrices above kSoloNMax: 2 x gvis_words
   long long gvis_words;
   unsigned long long* spill;  // oversize scratch: keys [0, cap), radix temp [cap, 2 cap)
+  int2* pend;                 // per output position: (row start, valence) of a node that did
+                              // not fit the ring, read back coalesced when it becomes a parent
+                              // (valence -1: not recorded, re-read row_ptr)
   long long spill_cap;
   Ctl* ctl;
   Stats* stats;
@@ -130,6 +137,8 @@ struct SoloMat {
   int nnz;
   uint32_t* vis;       // placed bitmap (smem or HBM)
   uint32_t* bvis;      // GL BFS bitmap (smem overlay or HBM)
+  int b0;              // bit of local node 0 in the first word (HBM bitmaps are packed
+                       // over all nodes, so neighbouring matrices may share a word)
   bool gmem;           // bitmaps in HBM
 };
 
@@ -212,30 +221,38 @@ __device__ __forceinline__ unsigned long long so_or_u64(unsigned long long v, So
 }
 
 __device__ __forceinline__ bool so_test(const SoloMat& M, int v) {
+  v += M.b0;
   const uint32_t w = M.gmem ? __ldcg(M.vis + (v >> 5)) : M.vis[v >> 5];
   return (w >> (v & 31)) & 1u;
 }
 template <bool kBig>
 __device__ __forceinline__ bool so_placed(const SoloMat& M, int v) {
   uint32_t w;
-  if constexpr (kBig) w = __ldcg(M.vis + (v >> 5));
+  if constexpr (kBig) { v += M.b0; w = __ldcg(M.vis + (v >> 5)); }
   else w = reinterpret_cast<const uint32_t*>(so_base() + kSoOffVis)[v >> 5];
   return (w >> (v & 31)) & 1u;
 }
-__device__ __forceinline__ void so_prefetch_l2(const void* p) {
-  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
-}
 __device__ __forceinline__ void so_set(const SoloMat& M, uint32_t* bits, int v) {
+  v += M.b0;
   atomicOr(bits + (v >> 5), 1u << (v & 31));
 }
 // test-and-set, true if this call set the bit
-__device__ __forceinline__ bool so_claim_bit(uint32_t* bits, int v) {
+__device__ __forceinline__ bool so_claim_bit(const SoloMat& M, uint32_t* bits, int v) {
+  v += M.b0;
   const uint32_t b = 1u << (v & 31);
   return !(atomicOr(bits + (v >> 5), b) & b);
 }
 
-__device__ __forceinline__ void so_zero_bits(uint32_t* bits, int n) {
-  for (int i = threadIdx.x; i < (n >> 5) + 1; i += kSoloNT) bits[i] = 0u;
+// Clear bits [b0, b0 + n): whole words with stores, a word shared with a
+// neighbouring matrix (HBM bitmaps) with an atomic AND of this matrix's bits.
+__device__ __forceinline__ void so_zero_bits(const SoloMat& M, uint32_t* bits) {
+  const int lo = M.b0, hi = M.b0 + M.n;       // bit range
+  const int w0 = lo >> 5, w1 = (hi - 1) >> 5;  // word range (inclusive)
+  for (int i = w0 + threadIdx.x; i <= w1; i += kSoloNT) {
+    const int bl = max(lo, i << 5) - (i << 5), bh = min(hi, (i << 5) + 32) - (i << 5);   // [bl, bh) in word i
+    if (bl == 0 && bh == 32) bits[i] = 0u;
+    else atomicAnd(bits + i, ~((bh == 32 ? 0xffffffffu : ((1u << bh) - 1u)) & ~((1u << bl) - 1u)));
+  }
 }
 
 __device__ __forceinline__ uint32_t so_hslot(uint32_t c) { return (c * 2654435761u) >> (32 - kSoloHBits); }
@@ -375,9 +392,9 @@ __device__ __forceinline__ int so_deg(const SoloMat& M, int v) { return __ldg(M.
 // Returns the number of levels; *minkey = min (valence, id) of the last level.
 static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long long* minkey, SoloSh& sh) {
   int32_t* q = M.perm;                        // entries [0, n - written) are free
-  so_zero_bits(M.bvis, M.n);
+  so_zero_bits(M, M.bvis);
   __syncthreads();
-  if (threadIdx.x == 0) { q[0] = r; so_claim_bit(M.bvis, r); sh.tail = 1; }
+  if (threadIdx.x == 0) { q[0] = r; so_claim_bit(M, M.bvis, r); sh.tail = 1; }
   __syncthreads();
   int head = 0, tail = 1, levels = 1;
   for (;;) {
@@ -385,7 +402,7 @@ static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long
       const int p = __ldcg(q + i);
       for (int e = __ldg(M.rp + p), ee = __ldg(M.rp + p + 1); e < ee; ++e) {
         const int c = __ldg(M.col + e);
-        if (so_claim_bit(M.bvis, c)) q[atomicAdd(&sh.tail, 1)] = c;
+        if (so_claim_bit(M, M.bvis, c)) q[atomicAdd(&sh.tail, 1)] = c;
       }
     }
     __syncthreads();
@@ -473,6 +490,8 @@ __device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& 
       so_ring_v()[q & (kSoloQ - 1)] = s;
       so_ring_rs()[q & (kSoloQ - 1)] = __ldg(M.rp + s);
       so_ring_d()[q & (kSoloQ - 1)] = so_deg(M, s);
+    } else if (kSoloPend) {
+      a.pend[M.node_base + q] = make_int2(0, -1);
     }
   }
   if (rhi == q) rhi = q + 1;
@@ -598,6 +617,7 @@ static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& 
     const int c = (int)(uint32_t)__ldcg(keys + i);
     M.perm[last - S.written - i] = c;
     if (a.iperm) a.iperm[M.node_base + c] = last - S.written - i;
+    if (!kBig && kSoloPend) a.pend[M.node_base + S.written + i] = make_int2(0, -1);   // row start not kept: re-read
   }
   if (threadIdx.x == 0) { ++sh.st_exec; ++sh.st_over; }
   S.pos += 1;
@@ -622,10 +642,11 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
     const int hi = min(S.written, S.pos + kSoloQ);
     for (int q = lo + t; q < hi; q += kSoloNT) {
       const int v = __ldcg(M.perm + last - q);
-      const int r0 = __ldg(M.rp + v);
+      int2 rd = (kBig || !kSoloPend) ? make_int2(0, -1) : __ldcg(a.pend + M.node_base + q);   // coalesced
+      if (rd.y < 0) { rd.x = __ldg(M.rp + v); rd.y = __ldg(M.rp + v + 1) - rd.x; }
       so_ring_v()[q & (kSoloQ - 1)] = v;
-      so_ring_rs()[q & (kSoloQ - 1)] = r0;
-      so_ring_d()[q & (kSoloQ - 1)] = __ldg(M.rp + v + 1) - r0;
+      so_ring_rs()[q & (kSoloQ - 1)] = rd.x;
+      so_ring_d()[q & (kSoloQ - 1)] = rd.y;
     }
     rhi = hi;
     if (!kBig) S.rhi = hi;
@@ -749,10 +770,13 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
     M.perm[last - q] = c;
     if (a.iperm) a.iperm[M.node_base + c] = last - q;
     if constexpr (!kBig) {
+      const int r0 = so_rsv()[key & 0x7fffu];
       if (ring_ok && q < pos_new + kSoloQ) {
         so_ring_v()[q & (kSoloQ - 1)] = c;
-        so_ring_rs()[q & (kSoloQ - 1)] = so_rsv()[key & 0x7fffu];
+        so_ring_rs()[q & (kSoloQ - 1)] = r0;
         so_ring_d()[q & (kSoloQ - 1)] = (int)(key >> 32);
+      } else if (kSoloPend) {
+        a.pend[M.node_base + q] = make_int2(r0, (int)(key >> 32));
       }
     }
   }
@@ -820,10 +844,11 @@ static __device__ void so_matrix(const SoloArgs& a, int k, SoloSh& sh) {
   M.col = a.col_idx + ci_base;
   M.perm = a.perm + M.node_base;
   M.gmem = M.n > kSoloNMax;
+  M.b0 = 0;
   if (M.gmem) {
-    const long long w = (M.node_base >> 5) + k;
-    M.vis = a.gvis + w;
-    M.bvis = a.gvis + a.gvis_words + w;
+    M.vis = a.gvis + (M.node_base >> 5);
+    M.bvis = a.gvis + a.gvis_words + (M.node_base >> 5);
+    M.b0 = (int)(M.node_base & 31);
   } else {
     M.vis = reinterpret_cast<uint32_t*>(so_base() + kSoOffVis);
     M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffCand);   // overlays the batch scratch
@@ -842,7 +867,7 @@ static __device__ void so_matrix(const SoloArgs& a, int k, SoloSh& sh) {
     const unsigned long long key = ((unsigned long long)(uint32_t)so_deg(M, v) << 32) | (uint32_t)v;
     best = key < best ? key : best;
   }
-  so_zero_bits(M.vis, M.n);
+  so_zero_bits(M, M.vis);
   // claim table starts empty (every batch restores it)
   if (!M.gmem) so_hash_reset<false>();
   else so_hash_reset<true>();

@@ -235,3 +235,23 @@ def test_hub_above_the_claims_bitmap(rcm):
     ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE)
     for path in ("default", "chain", "serial"):
         assert np.array_equal(_run(rcm, g, oracle.MIN_DEGREE, 0, **PATHS[path]), ref), path
+
+
+def test_batched_matrices_above_the_shared_bitmap(rcm):
+    """Matrices above 2^17 - 1 nodes keep their visited bitmaps in HBM, packed
+    over all nodes (neighbouring matrices share boundary words); with an
+    oversize hub and PSEUDO_PERIPHERAL."""
+    mats = [synth.relabel(synth.grid2d(400, 350), synth.randperm(140000, 11)), synth.path(37),
+            synth.relabel(synth.star(140000), synth.randperm(140001, 12)), synth.c5_matrix(5, 3000),
+            synth.relabel(synth.grid3d_27(53, 50, 50), synth.randperm(132500, 13))]
+    b = synth.batch_of(mats)
+    total, nnz = int(b.node_off[-1]), int(b.nnz_off[-1])
+    for mode in (oracle.MIN_DEGREE, oracle.PSEUDO_PERIPHERAL):
+        ref = oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, mode, threads=4)
+        plan = rcm.Plan(total, nnz, flags=rcm.RCM_FLAG_BATCHED_ONLY)
+        perm = plan.reorder_batched(_t(b.node_off), _t(b.nnz_off), _t(b.row_ptr_local), _t(b.col_idx_local),
+                                    total, nnz, mode=mode).cpu().numpy()
+        plan.close()
+        for k in range(len(mats)):
+            a0, a1 = int(b.node_off[k]), int(b.node_off[k + 1])
+            assert np.array_equal(perm[a0:a1], ref[a0:a1]), (mode, k)

@@ -1,11 +1,7 @@
 #!/bin/bash
-# One gpurun call: GPU tests, smoke, bench for every config, C2 launch list.
+# build, smoke, C5 timing (sweep_c5), all GPU tests, optional sanitizer
 mkdir -p gpurun_out
-nvidia-smi --query-gpu=name,driver_version,clocks.sm,clocks.max.sm --format=csv > gpurun_out/gpu.txt
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1
-timeout 1500 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1
-for c in 2 3 4 1; do
-  timeout 600 python bench.py --config $c --steps 10 --warmup 3 > gpurun_out/bench_c$c.json 2> gpurun_out/bench_c$c.err
-done
-timeout 900 python bench.py --config 5 --steps 5 --warmup 3 > gpurun_out/bench_c5.json 2> gpurun_out/bench_c5.err
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/c2_launches.csv python bench.py --config 2 --steps 2 --warmup 3 > gpurun_out/c2_ncu_bench.log 2>&1
+timeout 300 python tools/sweep_c5.py 5 > gpurun_out/sweep_now.jsonl 2> gpurun_out/sweep_now.err
+timeout 1500 python -m pytest tests -q -m gpu --timeout 300 --durations=15 ${PYTEST_ARGS} > gpurun_out/pytest_gpu.log 2>&1
+if [ -n "$SANITIZE" ]; then bash tools/gpu_sanitize.sh; fi
