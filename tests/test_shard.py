@@ -54,11 +54,12 @@ def _worker(rank, world, port, q):
     dist.destroy_process_group()
 
 
-def test_gather_two_ranks_gloo():
+@pytest.mark.parametrize("world", [2, 3])
+def test_gather_ranks_gloo(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
