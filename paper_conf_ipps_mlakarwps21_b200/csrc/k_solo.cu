@@ -10,7 +10,7 @@
 namespace rcm {
 
 #ifndef RCM_SOLO_MINB
-#define RCM_SOLO_MINB 4
+#define RCM_SOLO_MINB 5
 #endif
 
 __global__ void __launch_bounds__(1024) k_solo_order(const __grid_constant__ SoloArgs a) {

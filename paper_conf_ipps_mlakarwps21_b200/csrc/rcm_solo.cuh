@@ -41,10 +41,10 @@ namespace rcm {
 #define RCM_SOLO_NT 256
 #endif
 #ifndef RCM_SOLO_U
-#define RCM_SOLO_U 4
+#define RCM_SOLO_U 3
 #endif
 #ifndef RCM_SOLO_Q
-#define RCM_SOLO_Q 512
+#define RCM_SOLO_Q 256
 #endif
 #ifndef RCM_SOLO_PEND
 #define RCM_SOLO_PEND 1
@@ -64,7 +64,7 @@ constexpr int kSoloVisW = (kSoloNMax >> 5) + 1;     // bitmap words
 static_assert(kSoloT <= 32767 && (kSoloH & (kSoloH - 1)) == 0 && kSoloHBits <= 15, "claim table packing");
 static_assert((kSoloQ & (kSoloQ - 1)) == 0 && kSoloQ >= 256, "ring size");
 constexpr uint32_t kEmpty32 = 0xFFFFFFFFu;          // (c:17 | e:15) never reaches it: c < 2^17 - 1
-constexpr int kSoloGrp = 256;                       // output-group ring (stats only)
+constexpr int kSoloGrp = 64;                        // output-group ring (stats only)
 
 // Arguments of the solo kernels (one launch of k_solo_order + one of k_solo).
 struct SoloArgs {
@@ -99,15 +99,15 @@ struct SoloArgs {
 // Shared-memory layout (bytes), dynamic.
 constexpr size_t kSoOffVis = 0;
 constexpr size_t kSoOffRing = kSoOffVis + 4 * (size_t)kSoloVisW;
-constexpr size_t kSoOffPar = kSoOffRing + 12 * (size_t)kSoloQ;                 // 5 int arrays of kSoloNT + 1
-constexpr size_t kSoOffLpof = kSoOffPar + 5 * 4 * (size_t)(kSoloNT + 1) + 12;            // u16 per edge slot
+constexpr size_t kSoOffPar = kSoOffRing + 12 * (size_t)kSoloQ;                 // 3 int arrays of kSoloNT + 1
+constexpr size_t kSoOffLpof = kSoOffPar + 3 * 4 * (size_t)(kSoloNT + 1) + 4;             // u16 per edge slot
 constexpr size_t kSoOffFlp = kSoOffLpof + 2 * (size_t)kSoloT;                            // u16 per thread
 constexpr size_t kSoOffCand = (kSoOffFlp + 2 * (size_t)kSoloNT + 15) & ~size_t(15);
 constexpr size_t kSoOffHash = kSoOffCand + 8 * (size_t)kSoloT;
 constexpr size_t kSoOffRsv = kSoOffHash + 4 * (size_t)kSoloH;                  // big matrices: 8 B entries over hash+rsv
 constexpr size_t kSoOffRdeg = kSoOffRsv + 4 * (size_t)kSoloH;                 // valence per table slot
 constexpr size_t kSoloSmem = kSoOffRdeg + 4 * (size_t)kSoloH;
-static_assert(kSoloSmem - kSoOffCand >= 4 * (size_t)kSoloVisW, "GL bitmap overlays cand..rsv");
+static_assert(kSoloSmem - kSoOffRing >= 4 * (size_t)kSoloVisW, "GL bitmap overlays ring..rdeg");
 
 struct SoloSh {
   int32_t wtmp[kSoloNW + 1];
@@ -118,7 +118,6 @@ struct SoloSh {
   int32_t k, pos, written, rhi, nP, E, cnt, tail, found, big_n;
   int32_t cur_deg, cur_id, bad;
   unsigned long long minkey;
-  int32_t big_list[kSoloNT];
   long long st_exec, st_comp, st_over, st_claim, st_comb;
   // start positions of the pending output groups (one per batch), for the
   // work-aggregation counter: a batch whose parents span several groups
@@ -146,12 +145,15 @@ __device__ __forceinline__ uint8_t* so_base() { return rcm_dsm; }
 __device__ __forceinline__ int32_t* so_ring_v() { return reinterpret_cast<int32_t*>(so_base() + kSoOffRing); }
 __device__ __forceinline__ int32_t* so_ring_rs() { return so_ring_v() + kSoloQ; }
 __device__ __forceinline__ int32_t* so_ring_d() { return so_ring_v() + 2 * kSoloQ; }
-__device__ __forceinline__ int32_t* so_p_v() { return reinterpret_cast<int32_t*>(so_base() + kSoOffPar); }
-__device__ __forceinline__ int32_t* so_p_rs() { return so_p_v() + (kSoloNT + 1); }
-__device__ __forceinline__ int32_t* so_p_eo() { return so_p_v() + 2 * (kSoloNT + 1); }
-__device__ __forceinline__ int32_t* so_p_cnt() { return so_p_v() + 3 * (kSoloNT + 1); }
-__device__ __forceinline__ int32_t* so_p_pfx() { return so_p_v() + 4 * (kSoloNT + 1); }
+// per parent of the batch: row start, first edge slot (+ end), children filed
+__device__ __forceinline__ int32_t* so_p_rs() { return reinterpret_cast<int32_t*>(so_base() + kSoOffPar); }
+__device__ __forceinline__ int32_t* so_p_eo() { return so_p_rs() + (kSoloNT + 1); }
+__device__ __forceinline__ int32_t* so_p_cnt() { return so_p_rs() + 2 * (kSoloNT + 1); }
 __device__ __forceinline__ uint16_t* so_lpof() { return reinterpret_cast<uint16_t*>(so_base() + kSoOffLpof); }
+// segments above 16 children (sort phase), over the slot->parent table, which
+// is dead after the file phase
+__device__ __forceinline__ int32_t* so_big_list() { return reinterpret_cast<int32_t*>(so_base() + kSoOffLpof); }
+static_assert(2 * kSoloT >= 4 * kSoloNT || kSoloU < 2, "big-segment list overlays lpof");
 __device__ __forceinline__ uint16_t* so_flp() { return reinterpret_cast<uint16_t*>(so_base() + kSoOffFlp); }
 __device__ __forceinline__ unsigned long long* so_cand() {
   return reinterpret_cast<unsigned long long*>(so_base() + kSoOffCand);
@@ -660,7 +662,6 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   const int eo = so_scan1(d, sh.wscan[0], E);
   const bool fit = t < avail && eo + d <= kSoloT;
   if (fit) {
-    so_p_v()[t] = so_ring_v()[(pos + t) & (kSoloQ - 1)];
     so_p_rs()[t] = so_ring_rs()[(pos + t) & (kSoloQ - 1)];
     so_p_eo()[t] = eo;
     so_p_eo()[t + 1] = eo + d;   // == the next parent's offset; the last one ends the slots
@@ -744,7 +745,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
         seg[j + 1] = x;
       }
     } else {
-      sh.big_list[atomicAdd(&sh.nbig[par], 1)] = t;
+      so_big_list()[atomicAdd(&sh.nbig[par], 1)] = t;
     }
   }
   // ---- output positions: exclusive prefix of the per-parent counts
@@ -754,7 +755,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   if (nbig) {   // segments above 16 children: one warp each
     const int lane = t & 31, wid = t >> 5;
     for (int b = wid; b < nbig; b += kSoloNW) {
-      const int lp = sh.big_list[b];
+      const int lp = so_big_list()[b];
       bitonic_sort_flip(so_cand() + so_p_eo()[lp], so_p_cnt()[lp], lane, 32, [] { __syncwarp(); });
     }
     __syncthreads();
@@ -851,7 +852,9 @@ static __device__ void so_matrix(const SoloArgs& a, int k, SoloSh& sh) {
     M.b0 = (int)(M.node_base & 31);
   } else {
     M.vis = reinterpret_cast<uint32_t*>(so_base() + kSoOffVis);
-    M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffCand);   // overlays the batch scratch
+    // overlays the ring and the batch scratch: the GL finder runs only when no
+    // parent is pending (matrix start, component restart)
+    M.bvis = reinterpret_cast<uint32_t*>(so_base() + kSoOffRing);
   }
   if (a.validate && !so_validate(a, M, sh)) return;
   int seed;
