@@ -8,7 +8,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "librcm.so")
-SOURCES = ["rcm.cu", "k_main_inst.cu", "k_solo.cu", "k_probe.cu"]
+SOURCES = ["rcm.cu", "k_main_inst.cu", "k_solo.cu", "k_solo_sm.cu", "k_probe.cu"]
 HEADERS = ["rcm_device.cuh", "rcm_batch.cuh", "rcm_workers.cuh", "rcm_lookback.cuh", "rcm_components.cuh",
            "rcm_leveled.cuh", "rcm_main.cuh", "rcm_solo.cuh"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -57,6 +57,7 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None) ->
         extra = ["-Xptxas=-v", *extra]
     jobs = [(os.path.join(bdir, "rcm.o"), [os.path.join(CSRC, "rcm.cu")]),
             (os.path.join(bdir, "k_solo.o"), [os.path.join(CSRC, "k_solo.cu")]),
+            (os.path.join(bdir, "k_solo_sm.o"), [os.path.join(CSRC, "k_solo_sm.cu")]),
             (os.path.join(bdir, "k_probe.o"), [os.path.join(CSRC, "k_probe.cu")])]
     for bps, mb in KMAIN_VARIANTS:
         jobs.append((os.path.join(bdir, f"k_main_{bps}_{mb}.o"),

@@ -45,6 +45,7 @@ struct rcm_plan {
   int2* pend = nullptr;
   int solo_BS = 256;
   bool batched_only = false;
+  size_t smem_optin = 0;   // largest dynamic shared memory of one block
 };
 
 static rcm_status_t cuda_fail(cudaError_t e) {
@@ -102,6 +103,7 @@ extern "C" const void* rcm_ksolo_ptr();
 extern "C" size_t rcm_ksolo_smem();
 extern "C" int rcm_ksolo_threads();
 extern "C" int rcm_ksolo_nmax();
+extern "C" const void* rcm_ksolo_sm_ptr();
 static const void* pick_kernel(int bps, bool mb) {
   static_assert(1024 / kThreads >= 2, "two 512-thread blocks per SM");
   if (mb) return bps >= 2 ? rcm_kmain_ptr_2_1() : rcm_kmain_ptr_1_1();
@@ -188,6 +190,12 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, rcm_ksolo_ptr(), rcm_ksolo_threads(), p->solo_smem);
   if (occ_s <= 0) { delete p; return RCM_ERR_CUDA; }
   p->solo_blocks = occ_s * p->num_sms;
+  p->smem_optin = (size_t)smem_optin - 4096;   // room for the kernel's static shared memory
+  if (cudaFuncSetAttribute(rcm_ksolo_sm_ptr(), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem_optin) !=
+      cudaSuccess) {
+    delete p;
+    return RCM_ERR_CUDA;
+  }
   p->solo_BS = o.batch_nodes ? std::min(o.batch_nodes, rcm_ksolo_threads()) : rcm_ksolo_threads();
   p->mats_cap = n_max + 1;
   p->gvis_words = n_max / 32 + 2;   // bitmaps packed over all nodes (one bit each)
@@ -349,6 +357,19 @@ extern "C" rcm_status_t rcm_reorder(rcm_plan_t p, int32_t n, int64_t nnz, const 
     sa.nnz = nnz;
     sa.mode = (int)mode;
     sa.start = start;
+    // the whole CSR fits in shared memory next to the batch scratch: one block,
+    // no global round trip per batch (k_solo_sm)
+    const size_t csr = 4 * (((size_t)n + 1 + 3) / 4 * 4) + 4 * (size_t)nnz;
+    if (p->solo_smem + csr <= p->smem_optin && n <= rcm_ksolo_nmax()) {
+      sa.order = p->order; sa.gvis = p->gvis; sa.gvis_words = p->gvis_words; sa.spill = p->spill;
+      sa.spill_cap = p->spill_cap; sa.pend = p->pend; sa.ctl = p->ctl; sa.stats = p->stats;
+      sa.validate = p->opt.validate; sa.collect_stats = p->opt.collect_stats; sa.flags = p->opt.flags;
+      sa.BS = p->solo_BS;
+      void* args[] = {&sa};
+      CK(cudaLaunchKernel(rcm_ksolo_sm_ptr(), dim3(1), dim3(rcm_ksolo_threads()), args, p->solo_smem + csr,
+                          (cudaStream_t)stream));
+      return RCM_OK;
+    }
     return launch_solo(p, sa, (cudaStream_t)stream);
   }
   if (p->batched_only) return RCM_ERR_INVALID_ARGUMENT;   // no chain workspace in this plan

@@ -35,6 +35,14 @@
 #pragma once
 #include "rcm_batch.cuh"
 
+// Read-only CSR loads: through the non-coherent path from HBM, or plain loads
+// when the whole CSR of a small graph was staged in shared memory (k_solo_sm).
+#ifdef RCM_SOLO_SMEM_CSR
+#define SO_LD(p) (*(p))
+#else
+#define SO_LD(p) __ldg(p)
+#endif
+
 namespace rcm {
 
 #ifndef RCM_SOLO_NT
@@ -387,7 +395,7 @@ static __device__ void so_radix_sort_global(unsigned long long* a, unsigned long
 
 // --------------------------------------------------------------- seeds / GL
 // Valence of local node v.
-__device__ __forceinline__ int so_deg(const SoloMat& M, int v) { return __ldg(M.rp + v + 1) - __ldg(M.rp + v); }
+__device__ __forceinline__ int so_deg(const SoloMat& M, int v) { return SO_LD(M.rp + v + 1) - SO_LD(M.rp + v); }
 
 // Block-level BFS over the (wholly unplaced) component of r for the GL finder:
 // the queue lives in the not-yet-written part of perm, visited bits in M.bvis.
@@ -402,8 +410,8 @@ static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long
   for (;;) {
     for (int i = head + threadIdx.x; i < tail; i += kSoloNT) {
       const int p = __ldcg(q + i);
-      for (int e = __ldg(M.rp + p), ee = __ldg(M.rp + p + 1); e < ee; ++e) {
-        const int c = __ldg(M.col + e);
+      for (int e = SO_LD(M.rp + p), ee = SO_LD(M.rp + p + 1); e < ee; ++e) {
+        const int c = SO_LD(M.col + e);
         if (so_claim_bit(M, M.bvis, c)) q[atomicAdd(&sh.tail, 1)] = c;
       }
     }
@@ -490,7 +498,7 @@ __device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& 
     so_set(M, M.vis, s);
     if (rhi == q) {
       so_ring_v()[q & (kSoloQ - 1)] = s;
-      so_ring_rs()[q & (kSoloQ - 1)] = __ldg(M.rp + s);
+      so_ring_rs()[q & (kSoloQ - 1)] = SO_LD(M.rp + s);
       so_ring_d()[q & (kSoloQ - 1)] = so_deg(M, s);
     } else if (kSoloPend) {
       a.pend[M.node_base + q] = make_int2(0, -1);
@@ -505,12 +513,12 @@ __device__ __forceinline__ void so_place_root(const SoloArgs& a, const SoloMat& 
 // scan otherwise).  Returns true if the matrix is well formed.
 static __device__ bool so_validate(const SoloArgs& a, const SoloMat& M, SoloSh& sh) {
   int bad = 0;
-  if (threadIdx.x == 0) bad = (__ldg(M.rp) != 0) || (__ldg(M.rp + M.n) != M.nnz);
-  for (int v = threadIdx.x; v < M.n; v += kSoloNT) bad |= __ldg(M.rp + v + 1) < __ldg(M.rp + v);
+  if (threadIdx.x == 0) bad = (SO_LD(M.rp) != 0) || (SO_LD(M.rp + M.n) != M.nnz);
+  for (int v = threadIdx.x; v < M.n; v += kSoloNT) bad |= SO_LD(M.rp + v + 1) < SO_LD(M.rp + v);
   bad = __syncthreads_or(bad);
   if (!bad)
     for (int i = threadIdx.x; i < M.nnz; i += kSoloNT) {
-      const int c = __ldg(M.col + i);
+      const int c = SO_LD(M.col + i);
       bad |= (c < 0 || c >= M.n);
     }
   bad = __syncthreads_or(bad);
@@ -521,18 +529,18 @@ static __device__ bool so_validate(const SoloArgs& a, const SoloMat& M, SoloSh& 
   if (a.validate < 2) return true;
   int asym = 0;
   for (int u = threadIdx.x; u < M.n && !asym; u += kSoloNT) {   // thread per row
-    for (int e = __ldg(M.rp + u), re = __ldg(M.rp + u + 1); e < re && !asym; ++e) {
-      const int c = __ldg(M.col + e);
-      int lo = __ldg(M.rp + c), hi = __ldg(M.rp + c + 1) - 1;
+    for (int e = SO_LD(M.rp + u), re = SO_LD(M.rp + u + 1); e < re && !asym; ++e) {
+      const int c = SO_LD(M.col + e);
+      int lo = SO_LD(M.rp + c), hi = SO_LD(M.rp + c + 1) - 1;
       const int b0 = lo, b1 = hi;
       bool found = false;
       while (lo <= hi) {   // sorted row: O(log deg)
         const int mid = (lo + hi) >> 1;
-        const int x = __ldg(M.col + mid);
+        const int x = SO_LD(M.col + mid);
         if (x == u) { found = true; break; }
         if (x < u) lo = mid + 1; else hi = mid - 1;
       }
-      for (int f = b0; f <= b1 && !found; ++f) found = __ldg(M.col + f) == u;   // unsorted row
+      for (int f = b0; f <= b1 && !found; ++f) found = SO_LD(M.col + f) == u;   // unsorted row
       asym |= !found;
     }
   }
@@ -587,14 +595,14 @@ static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& 
 #pragma unroll
     for (int u = 0; u < kSoloU; ++u) {
       const int e = c0 + threadIdx.x * kSoloU + u;
-      cc[u] = e < D ? __ldg(M.col + rs + e) : -1;
+      cc[u] = e < D ? SO_LD(M.col + rs + e) : -1;
       ins[u] = false;
     }
 #pragma unroll
     for (int u = 0; u < kSoloU; ++u) {
       if (cc[u] >= 0 && !so_placed<kBig>(M, cc[u])) {
         slot[u] = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(threadIdx.x * kSoloU + u), &ins[u]);
-        if (ins[u]) { crs[u] = __ldg(M.rp + cc[u]); cre[u] = __ldg(M.rp + cc[u] + 1); }
+        if (ins[u]) { crs[u] = SO_LD(M.rp + cc[u]); cre[u] = SO_LD(M.rp + cc[u] + 1); }
       }
     }
     __syncthreads();
@@ -645,7 +653,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
     for (int q = lo + t; q < hi; q += kSoloNT) {
       const int v = __ldcg(M.perm + last - q);
       int2 rd = (kBig || !kSoloPend) ? make_int2(0, -1) : __ldcg(a.pend + M.node_base + q);   // coalesced
-      if (rd.y < 0) { rd.x = __ldg(M.rp + v); rd.y = __ldg(M.rp + v + 1) - rd.x; }
+      if (rd.y < 0) { rd.x = SO_LD(M.rp + v); rd.y = SO_LD(M.rp + v + 1) - rd.x; }
       so_ring_v()[q & (kSoloQ - 1)] = v;
       so_ring_rs()[q & (kSoloQ - 1)] = rd.x;
       so_ring_d()[q & (kSoloQ - 1)] = rd.y;
@@ -691,7 +699,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
       if (e < E) {
         while (so_p_eo()[lp + 1] <= e) ++lp;
         so_lpof()[e] = (uint16_t)lp;
-        cc[u] = __ldg(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
+        cc[u] = SO_LD(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
       }
     }
   }
@@ -702,9 +710,9 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
       bool ins;
       const int sl = so_claim<kBig>((uint32_t)cc[u], (uint32_t)(e0 + u), &ins);
       if (ins) {
-        const int r0 = __ldg(M.rp + cc[u]);
+        const int r0 = SO_LD(M.rp + cc[u]);
         if constexpr (!kBig) so_rsv()[sl] = r0;   // (big matrices: the 8 B entries overlay rsv)
-        so_rdeg()[sl] = __ldg(M.rp + cc[u] + 1) - r0;
+        so_rdeg()[sl] = SO_LD(M.rp + cc[u] + 1) - r0;
         slot[u] = sl;
       }
     }
