@@ -25,6 +25,7 @@ struct rcm_plan {
   int32_t* o = nullptr;
   Desc* desc = nullptr;
   Sig* sig = nullptr;
+  uint32_t* fwdv = nullptr;
   Ctl* ctl = nullptr;
   Stats* stats = nullptr;
   Problem* chains = nullptr;
@@ -78,7 +79,7 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->pend, p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->fwdv, p->pend, p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
                   p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
@@ -133,6 +134,7 @@ static rcm_status_t plan_alloc(rcm_plan* p) {
     AL(p->o, 4 * n);
     AL(p->desc, sizeof(Desc) * p->qcap);
     AL(p->sig, sizeof(Sig) * (p->qcap + 1));
+    AL(p->fwdv, 8 * (p->qcap + 1));
     AL(p->chains, sizeof(Problem) * p->prob_cap);
     AL(p->solos, sizeof(Problem) * p->prob_cap);
     if (o.collect_stats == 3) {
@@ -284,6 +286,7 @@ static KParams make_kparams(rcm_plan* p, const int32_t* row_ptr, const int32_t* 
   kp.dbg = p->dbg;
   kp.trace = p->trace;
   kp.trace_cap = p->trace_cap;
+  kp.fwdv = p->fwdv;
   return kp;
 }
 

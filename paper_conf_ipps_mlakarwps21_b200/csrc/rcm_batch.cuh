@@ -34,6 +34,7 @@ struct KParams {
   int32_t* dbg;               // per-block progress (8 ints per block), always written
   unsigned long long* trace;  // nullable: per-slot event times (collect_stats == 3)
   int32_t trace_cap;          // slots traced
+  uint32_t* fwdv;             // look-back chain, per slot that forwards its output: [2t] count, [2t+1] valence
 };
 
 // Per-slot event trace (collect_stats == 3), kTraceW words per slot:

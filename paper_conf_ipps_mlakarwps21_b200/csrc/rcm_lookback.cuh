@@ -24,11 +24,17 @@ namespace rcm {
 // Sig::word: Discovered flags, release stores (they order the block's
 // atomicMin marks, cumulatively, before the flag).
 constexpr unsigned long long LB_LOCAL = 1, LB_DINCL = 2;
+// set by a slot that forwarded its output once that output is written (the
+// receiver publishes batches over it only after seeing this flag)
+constexpr unsigned long long LB_OUTDONE = 4;
 // Sig::ovh holds the Counted facts, plain values (relaxed stores, no fence):
 //   AGG  = 2 | count << 2 (31 bit) | nb << 33 (30 bit)
 //   INCL = 1 | out_end << 2 (31 bit) | q_end << 33 (30 bit), replaces AGG
 // A successor reads one word per slot; nothing it reads depends on other data.
 constexpr unsigned long long LB_INCL = 1, LB_AGG = 2;
+// INCL bit 63: this slot forwarded its output to the next slot (work
+// aggregation); its count and valence sum are in KParams::fwdv
+constexpr unsigned long long LB_FWD = 1ull << 63;
 __device__ __forceinline__ unsigned long long lb_pfx(unsigned long long kind, long long a, long long b) {
   return kind | ((unsigned long long)(uint32_t)a << 2) | ((unsigned long long)(uint32_t)b << 33);
 }
@@ -128,7 +134,7 @@ static __device__ bool lb_prefix(const KParams& kp, const Problem& P, int t, int
       if (stop < 32) {
         const unsigned long long bs = __shfl_sync(0xffffffffu, b, stop);
         const int vs = __shfl_sync(0xffffffffu, (int)valid, stop);
-        if (vs) { base_out = (long long)((bs >> 2) & 0x7fffffffull); base_q = (long long)(bs >> 33); }
+        if (vs) { base_out = (long long)((bs >> 2) & 0x7fffffffull); base_q = (long long)((bs >> 33) & 0x3fffffffull); }
         j = -1;
         break;
       }
@@ -273,10 +279,53 @@ __device__ __forceinline__ int lb_phase_c(const KParams& kp, const Problem& P, c
         sh.out_off = out_off;
         sh.q_off = q_off;
         if ((long long)q_off + sh.nb > kp.qcap) { latch_error(kp.ctl, ST_CAPACITY); sh.nb = 0; sh.aborted = 1; }
-        st_relaxed_u64(&mine->ovh, lb_pfx(LB_INCL, out_off + sh.count, q_off + sh.nb));
+        // Work aggregation without a sequential decision chain: an
+        // even slot whose output is below half a batch (nodes and valence)
+        // forwards it to slot t+1 when t+1 is already a published non-empty
+        // batch; odd slots never forward, so an overhang is one slot deep and
+        // fits the receiver's first batch.  The receiver cuts the combined range
+        // into the slots both reserved (next-fit: NF(A ++ B) <= NF(A) + NF(B)).
+        bool fwd = false;
+        if (!(kp.flags & (F_NO_OVERHANG | F_MULTI_BATCH)) && !(t & 1) && !oversize && sh.count > 0 &&
+            2 * sh.count < kp.Bg && 2 * sh.V < (long long)kp.Tg && t + 1 < kp.qcap && !sh.aborted) {
+          const Desc* d1 = kp.desc + t + 1;
+          if (ld_acquire_u32(&d1->tag) == epoch)
+            fwd = ld_relaxed_s32(&d1->o_begin) < ld_relaxed_s32(&d1->o_end);
+        }
+        if (fwd) {
+          kp.fwdv[2 * t] = (uint32_t)sh.count;
+          kp.fwdv[2 * t + 1] = (uint32_t)sh.V;
+          __threadfence();
+          stat_add(kp, &kp.stats->ovh_forwards, 1);
+        }
+        sh.fwd = fwd;
+        st_relaxed_u64(&mine->ovh, lb_pfx(LB_INCL, out_off + sh.count, q_off + sh.nb) | (fwd ? LB_FWD : 0ull));
         atomicMax(&kp.ctl->qtail, q_off + sh.nb);
         atomicMax(&kp.ctl->chain_total, out_off + sh.count);
         stat_add(kp, &kp.stats->generated, sh.nb);
+        // receiver: an odd slot takes the overhang of slot t-1 if it forwarded
+        sh.ovh_n = 0;
+        sh.ovh_t = 0;
+        if ((t & 1) && !(kp.flags & (F_NO_OVERHANG | F_MULTI_BATCH)) && !sh.aborted) {
+          uint64_t t0 = 0;
+          for (int it = 0;; ++it) {
+            const unsigned long long b = ld_relaxed_u64(&kp.sig[t - 1].ovh);
+            if ((b & 3) == LB_AGG && ((b >> 2) & 0x7fffffffull) == 0) break;   // empty / no output: no forward
+            if ((b & 3) == LB_INCL) {
+              if (b & LB_FWD) {
+                fence_acquire_gpu();
+                sh.ovh_n = (int)__ldcg(kp.fwdv + 2 * (t - 1));
+                sh.ovh_t = (int)__ldcg(kp.fwdv + 2 * (t - 1) + 1);
+              }
+              break;
+            }
+            if (ld_relaxed_s32(&kp.ctl->done)) break;   // terminated: nothing left to batch
+            if ((it & 1023) == 1023) {
+              if (t0 == 0) t0 = globaltimer();
+              else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 7, t, (long long)b, 0); sh.aborted = 1; break; }
+            }
+          }
+        }
       } else {
         sh.aborted = 0;
       }
@@ -286,11 +335,20 @@ __device__ __forceinline__ int lb_phase_c(const KParams& kp, const Problem& P, c
   if (sh.aborted) return PH_ABORT;
   if (!sh.s_mid) return PH_C;
   clk_mark(kp, sh, 6);
-  const int out_off = sh.out_off, q_off = sh.q_off, nb = sh.nb;
+  const int out_off = sh.out_off;
+  // batches are cut over [out_off - overhang, out_off + count) into the slots
+  // reserved by the forwarder and by this batch (contiguous in the queue);
+  // a forwarder generates nothing and publishes none of its reserved slots
+  const int onb = sh.ovh_n > 0 ? lb_nb(kp, sh.ovh_n, sh.ovh_t) : 0;
+  const int q_off = sh.q_off - onb;
+  const int nb = sh.fwd ? 0 : sh.nb + onb;
   beacon(kp, 9, t, out_off);
   trace_ev(kp, t, 6);
   GenState g;
-  if (threadIdx.x == 0) { g.start = out_off; g.cnt = 0; g.val = 0; g.emitted = 0; g.has_pend = 0; g.defer = !oversize; }
+  if (threadIdx.x == 0) {
+    g.start = out_off - sh.ovh_n; g.cnt = sh.ovh_n; g.val = sh.ovh_t;
+    g.emitted = 0; g.has_pend = 0; g.defer = !oversize;
+  }
   if (oversize) {
     if (!oversize_gather_sort(kp, P, sm, sh, sm_p_rs(kp)[0], E)) return PH_ABORT;
     oversize_output(kp, P, sm, sh, out_off, nb > 0, g, q_off, nb, epoch);
@@ -319,9 +377,20 @@ __device__ __forceinline__ int lb_phase_c(const KParams& kp, const Problem& P, c
     }
     stat_add(kp, &kp.stats->executed, 1);
     const int total = out_off + sh.count;
+    if (sh.ovh_n > 0) {   // the forwarder's o[] entries must be visible before our batches cover them
+      uint64_t t0 = 0;
+      for (int it = 0; !(ld_relaxed_u64(&kp.sig[t - 1].word) & LB_OUTDONE); ++it) {
+        if (ld_relaxed_s32(&kp.ctl->done)) break;
+        if ((it & 1023) == 1023) {
+          if (t0 == 0) t0 = globaltimer();
+          else if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 8, t, 0, 0); break; }
+        }
+      }
+    }
     // one fence publishes the o[] writes and every descriptor's fields; the
     // tags (and the completion count) are then relaxed stores (release pattern)
     fence_acquire_gpu();
+    if (sh.fwd) st_relaxed_u64(&mine->word, LB_LOCAL | LB_DINCL | LB_OUTDONE);
     for (int i = 0; i < nb; ++i) st_relaxed_u32(&kp.desc[q_off + i].tag, epoch);
     if (total == P.pos0 + P.size) {             // early termination
       atomicExch(&kp.ctl->done, 1);
@@ -330,7 +399,7 @@ __device__ __forceinline__ int lb_phase_c(const KParams& kp, const Problem& P, c
       // reserves before it counts itself).  Fire-and-forget: chain end without
       // termination (completed == qtail) is detected by the idle dequeuers
       // (lb_chain_exhausted), off this block's critical path.
-      red_relaxed_add_s32(&kp.ctl->completed, 1 + (nb - emitted));
+      red_relaxed_add_s32(&kp.ctl->completed, 1 + (nb - emitted));   // a forwarder: nb = 0
     }
   }
   trace_ev(kp, t, 8);
