@@ -55,6 +55,12 @@ def _peaks():
     return HBM_FALLBACK_GBS, "fallback (B200_PROFILING.md)"
 
 
+def _dev_index(local_rank: int) -> int:
+    """GPU of this rank: LOCAL_RANK, or 0 for every rank when RCM_BENCH_SHARE_DEVICE=1
+    (testing the multi-rank harness on a single GPU with the gloo backend)."""
+    return 0 if os.environ.get("RCM_BENCH_SHARE_DEVICE") == "1" else local_rank
+
+
 def _cores() -> int:
     return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
 
@@ -219,6 +225,17 @@ def hop_probe(rcm, nsm: int, iters: int = 400):
         return {"unavailable": str(ex)[:120]}
 
 
+def _max_over_ranks(dist, x: float, dev) -> float:
+    """Max of a host float over all ranks (the device time of the slowest rank)."""
+    import torch
+    if dist is None:
+        return x
+    on_gpu = dist.get_backend() == "nccl"
+    t = torch.tensor([x], dtype=torch.float64, device=dev if on_gpu else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def time_events(fn, steps, stream, flush=None):
     import torch
     evs = []
@@ -266,11 +283,7 @@ def single_graph(rcm, cfg: int, steps: int, warmup: int, dev, world: int = 1, di
     sampler.start()
     ms_list = time_events(step, steps, stream, flush)
     clocks = sampler.stop()
-    dev_ms = sum(ms_list)
-    if dist is not None:
-        t = torch.tensor([dev_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dev_ms = float(t.item())
+    dev_ms = _max_over_ranks(dist, sum(ms_list), dev)
     if rcm.rcm_sync_status(plan.handle) != 0:
         raise RuntimeError("rcm_reorder failed")
     phases = plan.timing()
@@ -343,7 +356,7 @@ def run_c5(args, rank: int, world: int, local_rank: int, dist):
     import paper_conf_ipps_mlakarwps21_b200 as rcm
     from paper_conf_ipps_mlakarwps21_b200 import shard
 
-    dev = torch.device("cuda", local_rank)
+    dev = torch.device("cuda", _dev_index(local_rank))
     num = args.num_mats
     sizes = synth.c5_sizes(num)
     _, n_all, nnz_all = sd.c5_specs(np.arange(num), sizes)
@@ -377,7 +390,7 @@ def run_c5(args, rank: int, world: int, local_rank: int, dist):
     if dist is not None:
         dist.barrier()
     torch.cuda.synchronize()
-    sampler = ClockSampler(local_rank) if rank == 0 else None
+    sampler = ClockSampler(_dev_index(local_rank)) if rank == 0 else None
     if sampler:
         sampler.start()
     evs = []
@@ -438,11 +451,7 @@ def run_c5(args, rank: int, world: int, local_rank: int, dist):
             perm_h.copy_(perm, non_blocking=True)
             if world > 1:
                 gather()
-        e2e_ms = sum(time_events(e2e_step, e2e_steps, stream)) / e2e_steps
-        if dist is not None:
-            t = torch.tensor([e2e_ms], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_ms = float(t.item())
+        e2e_ms = _max_over_ranks(dist, sum(time_events(e2e_step, e2e_steps, stream)) / e2e_steps, dev)
         e2e = {"value": round(int(n_all.sum()) / (e2e_ms * 1e-3) / 1e6, 3), "unit": "Mnodes/s",
                "h2d_bytes_per_step": 4 * (rp_h.numel() + ci_h.numel()), "d2h_bytes_per_step": 4 * total,
                "ms_per_step": round(e2e_ms, 4), "steps": e2e_steps}
@@ -556,15 +565,19 @@ def main():
         run_reference(args, rank)
         return
     import torch
-    torch.cuda.set_device(local_rank)
+    torch.cuda.set_device(_dev_index(local_rank))
     dist = None
     if world > 1:
         import torch.distributed as dist
-        os.environ.setdefault("NCCL_DEBUG", "INFO")
-        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        backend = os.environ.get("RCM_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            dist.init_process_group("nccl", device_id=torch.device("cuda", _dev_index(local_rank)))
+        else:   # harness test of the multi-rank logic (gloo; ranks may share one GPU)
+            dist.init_process_group(backend)
     import paper_conf_ipps_mlakarwps21_b200 as rcm
-    dev = torch.device("cuda", local_rank)
+    dev = torch.device("cuda", _dev_index(local_rank))
     hop = hop_probe(rcm, torch.cuda.get_device_properties(dev).multi_processor_count) if rank == 0 else None
     if args.config == 5:
         line = run_c5(args, rank, world, local_rank, dist)

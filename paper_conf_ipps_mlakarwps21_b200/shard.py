@@ -30,15 +30,21 @@ def gather_to_root(local, part_sizes, rank: int, world: int, root: int = 0):
     import torch.distributed as dist
     if world == 1:
         return [local]
+    # NCCL moves device tensors over NVLink; gloo (CPU tests, harness checks)
+    # moves host copies
+    host = dist.get_backend() != "nccl" and local.is_cuda
+    buf = local.cpu() if host else local
     if rank == root:
-        out = [local if r == root else torch.empty(part_sizes[r], dtype=local.dtype, device=local.device)
+        out = [buf if r == root else torch.empty(part_sizes[r], dtype=local.dtype, device=buf.device)
                for r in range(world)]
         ops = [dist.P2POp(dist.irecv, out[r], r) for r in range(world) if r != root]
     else:
         out = None
-        ops = [dist.P2POp(dist.isend, local, root)]
+        ops = [dist.P2POp(dist.isend, buf, root)]
     for w in dist.batch_isend_irecv(ops):
         w.wait()
+    if host and out is not None:
+        out = [o.to(local.device) for o in out]
     return out
 
 
