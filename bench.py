@@ -215,12 +215,22 @@ def hop_probe(rcm, nsm: int, iters: int = 400):
         t = t[t > 0]
         if t.size < 4:
             return {"unavailable": "probe could not place blocks"}
-        thr = (t.min() + t.max()) / 2
-        near, far = t[t <= thr], t[t > thr]
-        return {"t_hop_ns_same_die": round(float(np.median(near)), 1),
-                "t_hop_ns_cross_die": round(float(np.median(far)), 1) if far.size else None,
-                "sm_pairs": int(t.size), "cross_die_pairs": int(far.size),
-                "how": f"SM0 -> SMj ping-pong, {iters} round trips, st.release.gpu / relaxed poll + fence.acq_rel"}
+        # two clusters (1-D 2-means): the two dies, if their hand-off latencies differ
+        lo, hi = float(t.min()), float(t.max())
+        for _ in range(20):
+            near = np.abs(t - lo) <= np.abs(t - hi)
+            if near.all() or (~near).all():
+                break
+            lo, hi = float(t[near].mean()), float(t[~near].mean())
+        near = np.abs(t - lo) <= np.abs(t - hi)
+        a, b = t[near], t[~near]
+        return {"t_hop_ns_same_die": round(float(np.median(a)), 1),
+                "t_hop_ns_cross_die": round(float(np.median(b)), 1) if b.size else None,
+                "sm_pairs": int(t.size), "cross_die_pairs": int(b.size),
+                "t_hop_ns_min_median_max": [round(float(t.min()), 1), round(float(np.median(t)), 1),
+                                            round(float(t.max()), 1)],
+                "how": f"SM0 -> SMj ping-pong, {iters} round trips, st.release.gpu / relaxed poll + fence.acq_rel; "
+                       "pairs split by 1-D 2-means"}
     except Exception as ex:
         return {"unavailable": str(ex)[:120]}
 

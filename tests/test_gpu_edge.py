@@ -255,3 +255,15 @@ def test_batched_matrices_above_the_shared_bitmap(rcm):
         for k in range(len(mats)):
             a0, a1 = int(b.node_off[k]), int(b.node_off[k + 1])
             assert np.array_equal(perm[a0:a1], ref[a0:a1]), (mode, k)
+
+
+def test_small_graph_with_a_large_csr(rcm):
+    """rcm_reorder on a graph of <= solo_threshold nodes whose CSR does not fit
+    in shared memory takes the global-memory one-block path (k_solo) instead
+    of the staged one (k_solo_sm); both must give the oracle's order."""
+    for g in (synth.complete(900), synth.gnp(3000, 0.05, 17, diag=True),
+              mutate.mutate(synth.gnp(2000, 0.08, 18), 19, **mutate.ALL["all"])):
+        assert 4 * (g.n + 1 + g.nnz) > 200 * 1024
+        for mode, s in ((oracle.FIXED, g.n // 3), (oracle.MIN_DEGREE, 0), (oracle.PSEUDO_PERIPHERAL, 0)):
+            ref = oracle.rcm(g.row_ptr, g.col_idx, mode, s)
+            assert np.array_equal(_run(rcm, g, mode, s), ref), (g.n, mode)
