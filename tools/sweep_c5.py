@@ -27,6 +27,12 @@ for k in sample:
     g = synth.c5_matrix(k, int(sizes[k]))
     a0, a1 = int(b["node_off_h"][k]), int(b["node_off_h"][k + 1])
     ok += np.array_equal(p[a0:a1], oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE))
+splan = rcm.Plan(b["total"], b["total_nnz"], flags=rcm.RCM_FLAG_BATCHED_ONLY, collect_stats=1)
+splan.reorder_batched(b["node_off"], b["nnz_off"], b["row_ptr_local"], b["col_idx_local"], b["total"], b["total_nnz"],
+                      perm_local=perm)
+st = splan.stats()
+splan.close()
 print(json.dumps({"lib": os.environ.get("RCM_LIB", "default"), "ms": round(statistics.median(ts), 3),
+                  "batches": st["batches_executed"], "combined": st["overhang_forwards"],
                   "min_ms": round(min(ts), 3), "solo_blocks": plan.info()["solo_blocks"],
                   "parity_sample": f"{ok}/{len(sample)}"}), flush=True)
