@@ -38,7 +38,7 @@ STATUS = {
 # every symbol include/rcm.h declares
 EXPORTS = ["rcm_default_options", "rcm_plan_create", "rcm_reorder", "rcm_reorder_batched",
            "rcm_find_pseudo_peripheral", "rcm_sync_status", "rcm_get_stats", "rcm_get_timing", "rcm_plan_info",
-           "rcm_plan_destroy", "rcm_status_string", "rcm_probe_hop"]
+           "rcm_plan_destroy", "rcm_status_string", "rcm_probe_hop", "rcm_reorder_batched_host"]
 
 
 class rcm_options_t(ctypes.Structure):
@@ -97,6 +97,8 @@ def _load():
     lib.rcm_get_timing.argtypes = [vp, ctypes.POINTER(ctypes.c_double)]
     lib.rcm_plan_destroy.argtypes = [vp]
     lib.rcm_plan_destroy.restype = None
+    lib.rcm_reorder_batched_host.argtypes = [vp, i32, vp, vp, vp, vp, i32, vp, vp, vp, vp, vp, vp, vp, vp, i32, vp]
+    lib.rcm_reorder_batched_host.restype = i32
     lib.rcm_probe_hop.argtypes = [i32, i32, i32, ctypes.POINTER(ctypes.c_double)]
     lib.rcm_probe_hop.restype = i32
     lib.rcm_status_string.argtypes = [i32]
@@ -175,6 +177,32 @@ def rcm_reorder_batched(plan, num_mats: int, total_nodes: int, total_nnz: int, n
         _ptr(col_idx_local, torch.int32, "col_idx_local"), int(mode), _ptr(starts, torch.int32, "starts"),
         _ptr(perm_local, torch.int32, "perm_local"), _stream(stream))
     _check(st, "rcm_reorder_batched")
+
+
+def _hptr(t, dtype, name):
+    """Host pointer of a CPU tensor (pinned for full PCIe bandwidth)."""
+    import torch
+    if t is None:
+        return None
+    if not isinstance(t, torch.Tensor) or t.is_cuda:
+        raise TypeError(f"{name} must be a CPU tensor")
+    if t.dtype != dtype or not t.is_contiguous():
+        raise TypeError(f"{name} must be a contiguous {dtype} tensor")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def rcm_reorder_batched_host(plan, num_mats: int, node_off_h, nnz_off_h, row_ptr_h, col_idx_h, mode: int,
+                             starts_h, perm_h, node_off_d, nnz_off_d, row_ptr_d, col_idx_d, starts_d, perm_d,
+                             chunks: int = 8, stream=None) -> None:
+    import torch
+    st = _load().rcm_reorder_batched_host(
+        plan, int(num_mats), _hptr(node_off_h, torch.int64, "node_off_h"), _hptr(nnz_off_h, torch.int64, "nnz_off_h"),
+        _hptr(row_ptr_h, torch.int32, "row_ptr_h"), _hptr(col_idx_h, torch.int32, "col_idx_h"), int(mode),
+        _hptr(starts_h, torch.int32, "starts_h"), _hptr(perm_h, torch.int32, "perm_h"),
+        _ptr(node_off_d, torch.int64, "node_off_d"), _ptr(nnz_off_d, torch.int64, "nnz_off_d"),
+        _ptr(row_ptr_d, torch.int32, "row_ptr_d"), _ptr(col_idx_d, torch.int32, "col_idx_d"),
+        _ptr(starts_d, torch.int32, "starts_d"), _ptr(perm_d, torch.int32, "perm_d"), int(chunks), _stream(stream))
+    _check(st, "rcm_reorder_batched_host")
 
 
 def rcm_find_pseudo_peripheral(plan, n: int, nnz: int, row_ptr, col_idx, start: int, out, stream=None):

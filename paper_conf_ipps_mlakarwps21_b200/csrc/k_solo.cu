@@ -17,16 +17,18 @@ __global__ void __launch_bounds__(1024) k_solo_order(const __grid_constant__ Sol
   __shared__ int32_t hist[33];
   if (threadIdx.x == 0) {
     Ctl* c = a.ctl;
-    c->ts[0] = globaltimer();
-    c->ts[1] = c->ts[0];
-    c->ts[2] = ~0ull;
-    c->ts[3] = c->ts[4] = c->ts[5] = c->ts[6] = 0;
-    c->status = 0;
     c->solo_next = 0;
-    c->done = 0;
-    c->n_chain = 0;
-    c->n_solo = 0;
-    if (a.collect_stats) *a.stats = Stats{};
+    if (a.chunk == 0) {
+      c->ts[0] = globaltimer();
+      c->ts[1] = c->ts[0];
+      c->ts[2] = ~0ull;
+      c->ts[3] = c->ts[4] = c->ts[5] = c->ts[6] = 0;
+      c->status = 0;
+      c->done = 0;
+      c->n_chain = 0;
+      c->n_solo = 0;
+      if (a.collect_stats) *a.stats = Stats{};
+    }
   }
   if (threadIdx.x < 33) hist[threadIdx.x] = 0;
   __syncthreads();

@@ -46,6 +46,7 @@ struct rcm_plan {
   int2* pend = nullptr;
   int solo_BS = 256;
   bool batched_only = false;
+  cudaStream_t s_copy = nullptr, s_kern = nullptr, s_back = nullptr;   // rcm_reorder_batched_host
   size_t smem_optin = 0;   // largest dynamic shared memory of one block
 };
 
@@ -88,6 +89,8 @@ static void free_all(rcm_plan* p) {
 
 extern "C" void rcm_plan_destroy(rcm_plan_t p) {
   if (!p) return;
+  for (cudaStream_t s : {p->s_copy, p->s_kern, p->s_back})
+    if (s) cudaStreamDestroy(s);
   free_all(p);
   delete p;
 }
@@ -248,6 +251,12 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
     // rcm_lookback.cuh lb_pfx): the queue never exceeds 2^30 - 1 slots
     p->qcap = std::min<int64_t>(o.queue_capacity ? o.queue_capacity : qb, (1ll << 30) - 1);
     p->prob_cap = std::max<int64_t>(1, n_max / 2 + 1);
+  }
+  if (cudaStreamCreateWithFlags(&p->s_copy, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&p->s_kern, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&p->s_back, cudaStreamNonBlocking) != cudaSuccess) {
+    rcm_plan_destroy(p);
+    return RCM_ERR_CUDA;
   }
   const rcm_status_t st = plan_alloc(p);
   if (st != RCM_OK) {
@@ -416,6 +425,92 @@ extern "C" rcm_status_t rcm_reorder_batched(rcm_plan_t p, int32_t num_mats, int6
   sa.num_mats = num_mats;
   sa.mode = (int)mode;
   return launch_solo(p, sa, (cudaStream_t)stream);
+}
+
+// Host-resident batch with copy/compute overlap: the batch is cut into
+// `chunks` ranges of matrices of about equal nnz; the H2D copy of range g+1
+// (copy stream) runs while range g is ordered (kernel stream), and range g's
+// permutations go back on a third stream.  Everything is ordered after the
+// work already enqueued on `stream`, and `stream` waits for all of it.
+extern "C" rcm_status_t rcm_reorder_batched_host(rcm_plan_t p, int32_t num_mats, const int64_t* node_off_h,
+                                                 const int64_t* nnz_off_h, const int32_t* row_ptr_h,
+                                                 const int32_t* col_idx_h, rcm_start_t mode, const int32_t* starts_h,
+                                                 int32_t* perm_h, int64_t* node_off_d, int64_t* nnz_off_d,
+                                                 int32_t* row_ptr_d, int32_t* col_idx_d, int32_t* starts_d,
+                                                 int32_t* perm_d, int32_t chunks, void* stream) {
+  if (!p || num_mats <= 0 || !node_off_h || !nnz_off_h || !row_ptr_h || !perm_h || !node_off_d || !nnz_off_d ||
+      !row_ptr_d || !perm_d || chunks <= 0)
+    return RCM_ERR_INVALID_ARGUMENT;
+  const int64_t total = node_off_h[num_mats], total_nnz = nnz_off_h[num_mats];
+  if (total < 0 || total_nnz < 0 || (total_nnz > 0 && (!col_idx_h || !col_idx_d))) return RCM_ERR_INVALID_ARGUMENT;
+  if (total > p->n_max || total_nnz > p->nnz_max || num_mats > p->mats_cap - 1) return RCM_ERR_INVALID_ARGUMENT;
+  if (mode < RCM_START_FIXED || mode > RCM_START_PSEUDO_PERIPHERAL) return RCM_ERR_INVALID_ARGUMENT;
+  if (mode == RCM_START_FIXED && (!starts_h || !starts_d)) return RCM_ERR_INVALID_ARGUMENT;
+  chunks = std::min(chunks, std::min<int32_t>(num_mats, 64));
+  cudaStream_t cs = p->s_copy, ks = p->s_kern, bs = p->s_back, us = (cudaStream_t)stream;
+  cudaEvent_t ev[2 * 64 + 4];
+  int nev = 0;
+  auto mk = [&]() -> cudaEvent_t {
+    cudaEvent_t e = nullptr;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    ev[nev++] = e;
+    return e;
+  };
+  cudaEvent_t e0 = mk();
+  CK(cudaEventRecord(e0, us));
+  CK(cudaStreamWaitEvent(cs, e0, 0));
+  CK(cudaStreamWaitEvent(ks, e0, 0));
+  CK(cudaStreamWaitEvent(bs, e0, 0));
+  CK(cudaMemcpyAsync(node_off_d, node_off_h, 8 * (size_t)(num_mats + 1), cudaMemcpyHostToDevice, cs));
+  CK(cudaMemcpyAsync(nnz_off_d, nnz_off_h, 8 * (size_t)(num_mats + 1), cudaMemcpyHostToDevice, cs));
+  if (starts_h && starts_d) CK(cudaMemcpyAsync(starts_d, starts_h, 4 * (size_t)num_mats, cudaMemcpyHostToDevice, cs));
+  int32_t m0 = 0;
+  for (int g = 0; g < chunks; ++g) {
+    // end of range g: the first matrix whose nnz prefix reaches (g+1)/chunks of the total
+    int32_t m1 = num_mats;
+    if (g + 1 < chunks) {
+      const int64_t target = total_nnz / chunks * (g + 1);
+      m1 = (int32_t)(std::lower_bound(nnz_off_h, nnz_off_h + num_mats + 1, target) - nnz_off_h);
+      m1 = std::max(m1, m0 + 1);
+      m1 = std::min(m1, num_mats - (chunks - 1 - g));
+    }
+    const int64_t r0 = node_off_h[m0] + m0, r1 = node_off_h[m1] + m1;   // row_ptr entries
+    const int64_t c0 = nnz_off_h[m0], c1 = nnz_off_h[m1];
+    CK(cudaMemcpyAsync(row_ptr_d + r0, row_ptr_h + r0, 4 * (size_t)(r1 - r0), cudaMemcpyHostToDevice, cs));
+    if (c1 > c0) CK(cudaMemcpyAsync(col_idx_d + c0, col_idx_h + c0, 4 * (size_t)(c1 - c0), cudaMemcpyHostToDevice, cs));
+    cudaEvent_t ec = mk();
+    CK(cudaEventRecord(ec, cs));
+    CK(cudaStreamWaitEvent(ks, ec, 0));
+    SoloArgs sa;
+    std::memset(&sa, 0, sizeof(sa));
+    sa.col_idx = col_idx_d;
+    sa.perm = perm_d;
+    sa.node_off = node_off_d + m0;
+    sa.nnz_off = nnz_off_d + m0;
+    sa.starts = starts_d ? starts_d + m0 : nullptr;
+    sa.num_mats = m1 - m0;
+    sa.mode = (int)mode;
+    sa.chunk = g;
+    // matrix k of the range is global matrix m0 + k: its row_ptr starts at
+    // node_off[m0 + k] + m0 + k -- shift the row_ptr base by m0 for the kernel's
+    // node_off[k] + k indexing
+    sa.row_ptr = row_ptr_d + m0;
+    const rcm_status_t st = launch_solo(p, sa, ks);
+    if (st != RCM_OK) return st;
+    cudaEvent_t ek = mk();
+    CK(cudaEventRecord(ek, ks));
+    CK(cudaStreamWaitEvent(bs, ek, 0));
+    const int64_t n0 = node_off_h[m0], n1 = node_off_h[m1];
+    if (n1 > n0) CK(cudaMemcpyAsync(perm_h + n0, perm_d + n0, 4 * (size_t)(n1 - n0), cudaMemcpyDeviceToHost, bs));
+    m0 = m1;
+  }
+  cudaEvent_t eb = mk(), ek = mk();
+  CK(cudaEventRecord(eb, bs));
+  CK(cudaEventRecord(ek, ks));
+  CK(cudaStreamWaitEvent(us, eb, 0));
+  CK(cudaStreamWaitEvent(us, ek, 0));
+  for (int i = 0; i < nev; ++i) cudaEventDestroy(ev[i]);   // released once completed
+  return RCM_OK;
 }
 
 extern "C" rcm_status_t rcm_find_pseudo_peripheral(rcm_plan_t p, int32_t n, int64_t nnz,

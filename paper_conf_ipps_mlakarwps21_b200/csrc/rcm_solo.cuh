@@ -102,6 +102,8 @@ struct SoloArgs {
   int collect_stats;
   int flags;
   int BS;                     // B_s (<= kSoloNT)
+  int chunk;                  // 0: a call's first launch (resets status, stats, timers);
+                              // > 0: a later chunk of rcm_reorder_batched_host
 };
 
 // Shared-memory layout (bytes), dynamic.

@@ -267,3 +267,33 @@ def test_small_graph_with_a_large_csr(rcm):
         for mode, s in ((oracle.FIXED, g.n // 3), (oracle.MIN_DEGREE, 0), (oracle.PSEUDO_PERIPHERAL, 0)):
             ref = oracle.rcm(g.row_ptr, g.col_idx, mode, s)
             assert np.array_equal(_run(rcm, g, mode, s), ref), (g.n, mode)
+
+
+@pytest.mark.parametrize("chunks", [1, 3, 8])
+def test_batched_host_pipeline(rcm, chunks):
+    """rcm_reorder_batched_host: host batch in, host permutations out, copies
+    overlapped with the ordering in `chunks` ranges; same result as the oracle
+    (and as the device API) for MIN_DEGREE, FIXED and PSEUDO_PERIPHERAL."""
+    mats = [synth.c5_matrix(k, n) for k, n in enumerate([1000, 2600, 1200, 4100, 900, 7000, 1500, 3300, 2000])]
+    mats.append(mutate.mutate(synth.c5_matrix(9, 1800), 5, **mutate.ALL["all"]))
+    b = synth.batch_of(mats)
+    num, total, nnz = len(mats), int(b.node_off[-1]), int(b.nnz_off[-1])
+    h = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731
+    starts = ((np.arange(num) * 7919) % np.diff(b.node_off)).astype(np.int32)
+    plan = rcm.Plan(total, nnz, flags=rcm.RCM_FLAG_BATCHED_ONLY)
+    for mode in (oracle.MIN_DEGREE, oracle.FIXED, oracle.PSEUDO_PERIPHERAL):
+        ref = oracle.rcm_batched(b.node_off, b.nnz_off, b.row_ptr_local, b.col_idx_local, mode,
+                                 starts if mode == oracle.FIXED else None)
+        perm_h = torch.empty(total, dtype=torch.int32).pin_memory()
+        dev = dict(node_off_d=torch.empty(num + 1, dtype=torch.int64, device="cuda"),
+                   nnz_off_d=torch.empty(num + 1, dtype=torch.int64, device="cuda"),
+                   row_ptr_d=torch.empty(b.row_ptr_local.size, dtype=torch.int32, device="cuda"),
+                   col_idx_d=torch.empty(nnz, dtype=torch.int32, device="cuda"),
+                   starts_d=torch.empty(num, dtype=torch.int32, device="cuda") if mode == oracle.FIXED else None,
+                   perm_d=torch.empty(total, dtype=torch.int32, device="cuda"))
+        rcm.rcm_reorder_batched_host(plan.handle, num, h(b.node_off), h(b.nnz_off), h(b.row_ptr_local),
+                                     h(b.col_idx_local), mode, h(starts) if mode == oracle.FIXED else None, perm_h,
+                                     chunks=chunks, **dev)
+        assert rcm.rcm_sync_status(plan.handle) == 0
+        assert np.array_equal(perm_h.numpy(), ref), (mode, chunks)
+    plan.close()
