@@ -30,7 +30,6 @@ struct rcm_plan {
   Stats* stats = nullptr;
   Problem* chains = nullptr;
   Problem* solos = nullptr;
-  unsigned long long* pm_key = nullptr;
   unsigned long long* spill = nullptr;
   int32_t* dbg = nullptr;
   unsigned long long* trace = nullptr;
@@ -80,9 +79,9 @@ extern "C" const char* rcm_status_string(rcm_status_t st) {
 }
 
 static void free_all(rcm_plan* p) {
-  void* ptrs[] = {p->fwdv, p->pend, p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->pm_key, p->spill,
+  void* ptrs[] = {p->fwdv, p->pend, p->order, p->gvis, p->trace, p->dbg, p->word, p->o, p->desc, p->sig, p->ctl, p->stats, p->chains, p->solos, p->spill,
                   p->w.label, p->w.ckey, p->w.csize, p->w.keys0, p->w.keys1, p->w.vals0, p->w.vals1,
-                  p->w.offs, p->w.hist, p->w.sctl, p->w.order, p->w.lev, p->w.front0, p->w.front1,
+                  p->w.offs, p->w.hist, p->w.sctl, p->w.lev, p->w.front0, p->w.front1,
                   p->w.gctl, p->w.gkey};
   for (void* q : ptrs) cudaFree(q);
 }

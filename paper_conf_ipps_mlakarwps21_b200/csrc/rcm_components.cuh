@@ -25,7 +25,6 @@ struct CompWS {
   long long* offs;             // component output offsets
   int32_t* hist;               // radix: 256 x tiles
   int32_t* sctl;               // [0] count, [1] current buffer, [2] skip flag
-  int32_t* order;              // batched: matrix order (LPT)
   int32_t* lev;                // GL levels
   int32_t* front0;
   int32_t* front1;
@@ -41,19 +40,11 @@ struct MainArgs {
   long long nnz;
   int mode;
   int start;
-  int solo;             // single graph: run as one solo problem
   int validate;
   int vec;              // row_ptr 16-byte aligned
   int thr;              // solo threshold for components
   long long prob_cap;
   int idbits;
-  int batched;
-  int num_mats;
-  long long total;
-  const int64_t* node_off;
-  const int64_t* nnz_off;
-  const int32_t* starts;
-  unsigned long long* pm_key;
   int gl_only;          // rcm_find_pseudo_peripheral
   int gl_start;
   int32_t* gl_out;

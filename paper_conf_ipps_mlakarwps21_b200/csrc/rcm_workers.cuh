@@ -44,31 +44,6 @@ static __device__ void grid_barrier(const KParams& kp) {
   __syncthreads();
 }
 
-// Unvisited node of minimum (valence, id) of a matrix (C-6), or -1.
-static __device__ int block_argmin_unvisited(const KParams& kp, const Problem& P, ShState& sh) {
-  unsigned long long best = kKeyMax;
-  const unsigned long long* word = kp.word + P.node_base;
-  for (int v = threadIdx.x; v < P.mat_n; v += kThreads) {
-    unsigned long long w = ld_relaxed_u64(word + v);
-    if ((uint32_t)(w >> 32) == kInf) {
-      unsigned long long k = ((w & 0xffffffffull) << 32) | (uint32_t)v;
-      best = k < best ? k : best;
-    }
-  }
-  best = warp_min_u64(best);
-  if ((threadIdx.x & 31) == 0) sh.wtmp64[threadIdx.x >> 5] = best;
-  __syncthreads();
-  if (threadIdx.x < 32) {
-    unsigned long long b = threadIdx.x < kWarps ? sh.wtmp64[threadIdx.x] : kKeyMax;
-    b = warp_min_u64(b);
-    if (threadIdx.x == 0) sh.minkey = b;
-  }
-  __syncthreads();
-  unsigned long long r = sh.minkey;
-  __syncthreads();
-  return r == kKeyMax ? -1 : (int)(uint32_t)r;
-}
-
 // ---------------------------------------------------- block radix sort (global)
 // Stable LSD radix sort (8-bit digits) of a[0..n) in global memory by one
 // block, temp buffer tmp[0..n); digits that are equal in all keys are skipped.
@@ -651,9 +626,9 @@ static __device__ int block_gl(const KParams& kp, const Problem& P, int32_t* q, 
   }
 }
 
-// One block orders a whole component (or a whole small matrix, restarting at
-// the C-6 seed when a component is exhausted) with the same batch steps but
-// without the signalling chain: batches are consecutive output ranges.
+// One block orders a whole (small) component of a large graph with the same
+// batch steps but without the signalling chain: batches are consecutive output
+// ranges.  (Batched matrices and small graphs use rcm_solo.cuh instead.)
 __device__ __forceinline__ void run_solo(const KParams& kp, const Problem& P, const SmemPtrs& sm, ShState& sh, int32_t* lev) {
   int seed = P.seed;
   if (P.flags & 2) seed = block_gl(kp, P, kp.o + P.o_base + P.pos0, lev, seed, sh);
@@ -668,23 +643,10 @@ __device__ __forceinline__ void run_solo(const KParams& kp, const Problem& P, co
   for (;;) {
     if (pos == written) {
       if (written >= end) break;
-      if (!(P.flags & 1)) {          // declared size larger than the component
-        if (threadIdx.x == 0) latch_error(kp.ctl, ST_NOT_SYM);
-        break;
-      }
-      int s = block_argmin_unvisited(kp, P, sh);
-      if (s < 0) {
-        if (threadIdx.x == 0) latch_error(kp.ctl, ST_BAD_CSR);
-        break;
-      }
-      if (P.flags & 2) s = block_gl(kp, P, kp.o + P.o_base + written, lev, s, sh);
-      if (threadIdx.x == 0) {
-        place_root(kp, P, s, written);
-        stat_add(kp, &kp.stats->components, 1);
-      }
-      ++written;
-      __syncthreads();
-      continue;
+      // a component problem whose declared size exceeds what its BFS reaches:
+      // the pattern is not symmetric (C-9)
+      if (threadIdx.x == 0) latch_error(kp.ctl, ST_NOT_SYM);
+      break;
     }
     int nP = load_parents(kp, P, sm, sh, pos, min(kp.BS, written - pos), true);
     const int E = sh.E;
