@@ -428,39 +428,46 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
   const int G = gthreads(kp);
   const int lane = threadIdx.x & 31;
   const int gwarp = gtid() >> 5, nwarps = G >> 5;
+  // per-level counters rotate over three slots (frontier size, warp-row list,
+  // block-row list at gctl[8 + i], [12 + i], [16 + i]): level L counts into
+  // slot L % 3 and clears slot (L + 1) % 3, last read before the barrier of
+  // level L - 1 -- one grid barrier per level
+  int32_t* cnt = w.gctl + 8;
+  int32_t* cmed = w.gctl + 12;
+  int32_t* cbig = w.gctl + 16;
   for (int v = gtid(); v < n; v += G) w.lev[v] = -1;
   grid_barrier(kp);
   if (gtid() == 0) {
     w.lev[r] = 0;
     w.front0[0] = r;
-    w.gctl[0] = 0;
-    w.gctl[4] = 0;
-    w.gctl[5] = 0;
+    cnt[0] = cmed[0] = cbig[0] = 0;
     w.gkey[0] = kKeyMax;
   }
   grid_barrier(kp);
   int32_t* cur = w.front0;
   int32_t* nxt = w.front1;
   int ncur = 1, level = 0;
-  auto visit = [&](int c) {
-    if (ld_cg_s32(w.lev + c) < 0 && atomicCAS(w.lev + c, -1, level + 1) == -1) nxt[atomicAdd(w.gctl, 1)] = c;
-  };
   for (;;) {
+    const int sl = level % 3;
+    if (gtid() == 0) { const int s1 = (level + 1) % 3; cnt[s1] = 0; cmed[s1] = 0; cbig[s1] = 0; }
+    auto visit = [&](int c) {
+      if (ld_cg_s32(w.lev + c) < 0 && atomicCAS(w.lev + c, -1, level + 1) == -1) nxt[atomicAdd(cnt + sl, 1)] = c;
+    };
     // rows up to 32 entries: one thread; longer rows are listed for a warp
     // (vals0) or, above 4096 entries, a whole block (vals1), so hub rows are split
     for (int i = gtid(); i < ncur; i += G) {
       const int p = __ldcg(cur + i);
       const int rs = __ldg(kp.row_ptr + p), re = __ldg(kp.row_ptr + p + 1);
       if (re - rs > 32) {
-        if (re - rs > 4096) w.vals1[atomicAdd(w.gctl + 5, 1)] = p;
-        else w.vals0[atomicAdd(w.gctl + 4, 1)] = p;
+        if (re - rs > 4096) w.vals1[atomicAdd(cbig + sl, 1)] = p;
+        else w.vals0[atomicAdd(cmed + sl, 1)] = p;
         continue;
       }
       for (int e = rs; e < re; ++e) visit(__ldg(kp.col_idx + e));
     }
     grid_barrier(kp);
-    const int nmed = ld_cg_s32(w.gctl + 4), nbig = ld_cg_s32(w.gctl + 5);
-    if (nmed | nbig) {   // block-uniform: read after the barrier
+    const int nmed = ld_cg_s32(cmed + sl), nbig = ld_cg_s32(cbig + sl);
+    if (nmed | nbig) {   // uniform: read after the barrier
       for (int i = gwarp; i < nmed; i += nwarps) {
         const int p = __ldcg(w.vals0 + i);
         for (int e = __ldg(kp.row_ptr + p) + lane; e < __ldg(kp.row_ptr + p + 1); e += 32) visit(__ldg(kp.col_idx + e));
@@ -472,14 +479,11 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
       }
       grid_barrier(kp);
     }
-    const int nn = ld_cg_s32(w.gctl);
-    grid_barrier(kp);
+    const int nn = ld_cg_s32(cnt + sl);
     if (nn == 0) break;
-    if (gtid() == 0) { w.gctl[0] = 0; w.gctl[4] = 0; w.gctl[5] = 0; }
     ++level;
     int32_t* t = cur; cur = nxt; nxt = t;
     ncur = nn;
-    grid_barrier(kp);
   }
   unsigned long long best = kKeyMax;
   for (int i = gtid(); i < ncur; i += G) {
