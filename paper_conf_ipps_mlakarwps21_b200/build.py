@@ -37,7 +37,7 @@ def _extra_defines() -> list:
         extra.append(f"-DRCM_DISC_U={os.environ['RCM_DISC_U']}")
     if os.environ.get("RCM_TRACE"):
         extra.append("-DRCM_TRACE")
-    for k in ("RCM_SOLO_U", "RCM_SOLO_Q", "RCM_SOLO_NT", "RCM_SOLO_MINB", "RCM_SOLO_PEND", "RCM_SOLO_PIPE"):   # solo-path variants (sweeps)
+    for k in ("RCM_SOLO_U", "RCM_SOLO_Q", "RCM_SOLO_NT", "RCM_SOLO_MINB", "RCM_SOLO_PEND", "RCM_SOLO_PIPE", "RCM_DQ_SLEEP_MAX", "RCM_LB_SLEEP_MAX", "RCM_CC_SAMPLE"):   # solo-path variants (sweeps)
         if os.environ.get(k):
             extra.append(f"-D{k}={os.environ[k]}")
     return extra

@@ -347,6 +347,10 @@ static __device__ void signal_count(const KParams& kp, ShState& sh, const Sig* m
 // exactly once, so completed == qtail read in this order (acquire) implies no
 // slot is still running.  Polled by blocks idling in dequeue.
 static __device__ __noinline__ bool lb_chain_exhausted(const KParams& kp) {
+  // relaxed polls first: an ld.acquire.gpu invalidates the whole SM's L1 (the
+  // other resident block's cached rows included), so idle blocks only pay for
+  // the acquire when the counters look equal
+  if (ld_relaxed_s32(&kp.ctl->completed) != ld_relaxed_s32(&kp.ctl->qtail)) return false;
   const int c = ld_acquire_s32(&kp.ctl->completed);
   if (c != ld_acquire_s32(&kp.ctl->qtail)) return false;
   kp.ctl->incomplete = 1;   // idempotent: several idle blocks may get here
