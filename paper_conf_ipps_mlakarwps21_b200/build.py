@@ -17,7 +17,7 @@ FLAGS = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-
          "-Xptxas", "-warn-spills"]
 # one translation unit per persistent-kernel variant (compiled in parallel):
 # (min blocks per SM, multi-batch execution)
-KMAIN_VARIANTS = [(2, 0), (1, 0), (2, 1), (1, 1)]
+KMAIN_VARIANTS = [(2, 0), (1, 0), (2, 1), (1, 1), (2, 2), (1, 2)]   # (blocks per SM, 0 chain / 1 multi-batch / 2 leveled)
 BUILD_DIR = os.path.join(HERE, "..", "build", "obj")
 
 

@@ -96,19 +96,22 @@ extern "C" void rcm_plan_destroy(rcm_plan_t p) {
 
 // k_main instantiations (k_main_inst.cu, one translation unit each): 1 or 2
 // resident blocks per SM (register budget 64K / (bps * kThreads)), with or
-// without multi-batch execution.
+// traversal mode 0 chain / 1 multi-batch chain / 2 leveled.
 extern "C" const void* rcm_kmain_ptr_1_0();
 extern "C" const void* rcm_kmain_ptr_2_0();
 extern "C" const void* rcm_kmain_ptr_1_1();
 extern "C" const void* rcm_kmain_ptr_2_1();
+extern "C" const void* rcm_kmain_ptr_1_2();
+extern "C" const void* rcm_kmain_ptr_2_2();
 extern "C" const void* rcm_ksolo_order_ptr();
 extern "C" const void* rcm_ksolo_ptr();
 extern "C" size_t rcm_ksolo_smem();
 extern "C" int rcm_ksolo_threads();
 extern "C" int rcm_ksolo_nmax();
 extern "C" const void* rcm_ksolo_sm_ptr();
-static const void* pick_kernel(int bps, bool mb) {
+static const void* pick_kernel(int bps, bool mb, bool lv) {
   static_assert(1024 / kThreads >= 2, "two 512-thread blocks per SM");
+  if (lv) return bps >= 2 ? rcm_kmain_ptr_2_2() : rcm_kmain_ptr_1_2();
   if (mb) return bps >= 2 ? rcm_kmain_ptr_2_1() : rcm_kmain_ptr_1_1();
   return bps == 2 ? rcm_kmain_ptr_2_0() : rcm_kmain_ptr_1_0();
 }
@@ -234,7 +237,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
     p->T = T;
     p->smem = nctx == 1 ? smem_bytes(p->BS, T) : nctx * ((smem_bytes(p->BS, T) + 15) & ~size_t(15));
     // one block per SM: the 128-register build (no spills); more: the 64-register build
-    p->kernel = pick_kernel(bps, nctx == 2);
+    p->kernel = pick_kernel(bps, nctx == 2, (o.flags & RCM_FLAG_LEVELED) != 0);
     if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {
       delete p;
       return RCM_ERR_CUDA;

@@ -113,6 +113,7 @@ __host__ __device__ inline size_t smem_bytes(int BS, int T) {
 }
 
 // Static shared state of one worker.
+constexpr int kLvList = 32;   // leveled traversal: output regions per block and round
 struct ShState {
   unsigned long long wtmp64[kWarps + 1];
   long long wtmp64b[kWarps + 1];
@@ -131,6 +132,7 @@ struct ShState {
   int64_t spill_base;
   uint32_t* ovbits;            // oversize claims bitmap (shared memory, or HBM scratch for long rows)
   int32_t big_list[256];
+  int32_t lv_off[kLvList], lv_cnt[kLvList], lv_n;   // leveled traversal: this block's output list
   long long clk[10];           // per-stage cycle accumulators (thread 0)
   long long tclk;
   Problem prob;                // the problem being traversed (chain or solo)

@@ -9,6 +9,7 @@
 
 #include "../../include/rcm.h"
 #include "rcm_lookback.cuh"
+#include "rcm_expand.cuh"
 
 namespace rcm {
 
@@ -428,19 +429,20 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
   const int G = gthreads(kp);
   const int lane = threadIdx.x & 31;
   const int gwarp = gtid() >> 5, nwarps = G >> 5;
-  // per-level counters rotate over three slots (frontier size, warp-row list,
-  // block-row list at gctl[8 + i], [12 + i], [16 + i]): level L counts into
-  // slot L % 3 and clears slot (L + 1) % 3, last read before the barrier of
-  // level L - 1 -- one grid barrier per level
+  constexpr int kU = 4;          // edges per lane in flight
+  constexpr int kChunk = 1024;   // rows longer than this are split into kChunk-edge items, one warp each
+  // per-level counters rotate over three slots (next-frontier size, long-row
+  // items at gctl[8 + i], [16 + i]): level L counts into slot L % 3 and clears
+  // slot (L + 1) % 3, last read before the barrier of level L - 1 -- one grid
+  // barrier per level (two when the level has rows above kChunk)
   int32_t* cnt = w.gctl + 8;
-  int32_t* cmed = w.gctl + 12;
   int32_t* cbig = w.gctl + 16;
   for (int v = gtid(); v < n; v += G) w.lev[v] = -1;
   grid_barrier(kp);
   if (gtid() == 0) {
     w.lev[r] = 0;
     w.front0[0] = r;
-    cnt[0] = cmed[0] = cbig[0] = 0;
+    cnt[0] = cbig[0] = 0;
     w.gkey[0] = kKeyMax;
   }
   grid_barrier(kp);
@@ -449,33 +451,81 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
   int ncur = 1, level = 0;
   for (;;) {
     const int sl = level % 3;
-    if (gtid() == 0) { const int s1 = (level + 1) % 3; cnt[s1] = 0; cmed[s1] = 0; cbig[s1] = 0; }
-    auto visit = [&](int c) {
-      if (ld_cg_s32(w.lev + c) < 0 && atomicCAS(w.lev + c, -1, level + 1) == -1) nxt[atomicAdd(cnt + sl, 1)] = c;
-    };
-    // rows up to 32 entries: one thread; longer rows are listed for a warp
-    // (vals0) or, above 4096 entries, a whole block (vals1), so hub rows are split
-    for (int i = gtid(); i < ncur; i += G) {
-      const int p = __ldcg(cur + i);
-      const int rs = __ldg(kp.row_ptr + p), re = __ldg(kp.row_ptr + p + 1);
-      if (re - rs > 32) {
-        if (re - rs > 4096) w.vals1[atomicAdd(cbig + sl, 1)] = p;
-        else w.vals0[atomicAdd(cmed + sl, 1)] = p;
-        continue;
+    if (gtid() == 0) { const int s1 = (level + 1) % 3; cnt[s1] = 0; cbig[s1] = 0; }
+    // the kU column loads of a lane, then kU level loads, then the CASes; the
+    // newly reached nodes are appended with one atomicAdd per warp and round
+    auto visit = [&](const int (&c)[kU]) {
+      int lv[kU];
+#pragma unroll
+      for (int u = 0; u < kU; ++u) lv[u] = c[u] >= 0 ? ld_cg_s32(w.lev + c[u]) : 0;
+      bool nw[kU];
+      int k = 0;
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+        nw[u] = c[u] >= 0 && lv[u] < 0 && atomicCAS(w.lev + c[u], -1, level + 1) == -1;
+        k += nw[u];
       }
-      for (int e = rs; e < re; ++e) visit(__ldg(kp.col_idx + e));
+      const int incl = warp_incl_scan(k);
+      const int tot = __shfl_sync(kFull, incl, 31);
+      if (tot) {
+        int base = 0;
+        if (lane == 31) base = atomicAdd(cnt + sl, tot);
+        base = __shfl_sync(kFull, base, 31) + incl - k;
+#pragma unroll
+        for (int u = 0; u < kU; ++u)
+          if (nw[u]) nxt[base++] = c[u];
+      }
+    };
+    // frontier nodes per warp: spread a narrow level over all warps
+    const int per = min(32, max(1, (ncur + nwarps - 1) / nwarps));
+    for (int i0 = gwarp * per; i0 < ncur; i0 += nwarps * per) {
+      const int i = i0 + lane;
+      int p = -1, rs = 0, d = 0;
+      if (lane < per && i < ncur) {
+        p = __ldcg(cur + i);
+        rs = __ldg(kp.row_ptr + p);
+        d = __ldg(kp.row_ptr + p + 1) - rs;
+      }
+      const int nit = d > kChunk ? (d + kChunk - 1) / kChunk : 0;   // long row -> items
+      const int iincl = warp_incl_scan(nit);
+      const int itot = __shfl_sync(kFull, iincl, 31);
+      if (itot) {
+        int base = 0;
+        if (lane == 31) base = atomicAdd(cbig + sl, itot);
+        base = __shfl_sync(kFull, base, 31);
+        if (base + itot > w.cap) {
+          if (lane == 0) latch_error(kp.ctl, ST_CAPACITY);
+        } else {
+          for (int k = 0; k < nit; ++k) {
+            w.vals0[base + iincl - nit + k] = p;
+            w.vals1[base + iincl - nit + k] = k;
+          }
+        }
+      }
+      WarpRows R;
+      R.init(rs, nit ? 0 : d);
+      for (int b = 0; b < R.E; b += 32 * kU) {
+        int c[kU], j[kU];
+        R.cols<kU>(kp.col_idx, b, c, j);
+        visit(c);
+      }
     }
     grid_barrier(kp);
-    const int nmed = ld_cg_s32(cmed + sl), nbig = ld_cg_s32(cbig + sl);
-    if (nmed | nbig) {   // uniform: read after the barrier
-      for (int i = gwarp; i < nmed; i += nwarps) {
-        const int p = __ldcg(w.vals0 + i);
-        for (int e = __ldg(kp.row_ptr + p) + lane; e < __ldg(kp.row_ptr + p + 1); e += 32) visit(__ldg(kp.col_idx + e));
-      }
-      for (int i = blockIdx.x; i < nbig; i += kp.nblocks) {
-        const int p = __ldcg(w.vals1 + i);
-        for (int e = __ldg(kp.row_ptr + p) + threadIdx.x; e < __ldg(kp.row_ptr + p + 1); e += kThreads)
-          visit(__ldg(kp.col_idx + e));
+    const int nbig = ld_cg_s32(cbig + sl);
+    if (nbig) {   // uniform: read after the barrier
+      for (int it = gwarp; it < nbig; it += nwarps) {
+        const int p = __ldcg(w.vals0 + it), k = __ldcg(w.vals1 + it);
+        const int rs = __ldg(kp.row_ptr + p) + k * kChunk;
+        const int re = min(__ldg(kp.row_ptr + p + 1), rs + kChunk);
+        for (int b = rs; b < re; b += 32 * kU) {
+          int c[kU];
+#pragma unroll
+          for (int u = 0; u < kU; ++u) {
+            const int e = b + u * 32 + lane;
+            c[u] = e < re ? __ldg(kp.col_idx + e) : -1;
+          }
+          visit(c);
+        }
       }
       grid_barrier(kp);
     }

@@ -1,6 +1,6 @@
 // rcm_main.cuh -- the persistent kernel k_main (one cooperative launch per
 // rcm_* call) and its phases: prologue, seeding, traversal scheduling,
-// components.  Instantiated once per (blocks-per-SM, multi-batch) variant in
+// components.  Instantiated once per (blocks-per-SM, chain / multi-batch / leveled) variant in
 // k_main_inst.cu (separate translation units, compiled in parallel).
 // Citations P:L<n> = /root/reference/PAPER.md line n; C-k = DESIGN.md readings.
 #pragma once
@@ -96,7 +96,9 @@ static __device__ void validate_sym_phase(const KParams& kp, int n) {
 
 // The scheduling phase: every chain problem in turn on all blocks (grid
 // barrier between chains), then the solo problems, one per block at a time.
-template <bool kMB>
+// kMode: 0 look-back / serial chain, 1 multi-batch chain, 2 leveled (NEXT-3);
+// one kernel instantiation each, so no variant pays the others' registers.
+template <int kMode>
 __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs& a, const SmemPtrs& sm, ShState& sh,
                                                ShState& sh2) {
   const int nchain = ld_cg_s32(&kp.ctl->n_chain);
@@ -106,7 +108,7 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
       if (blockIdx.x == 0 && threadIdx.x == 0) const_cast<Problem*>(kp.chains)[c].seed = x;
       grid_barrier(kp);
     }
-    if (kp.flags & F_LEVELED) {      // NEXT-3: Alg. 2 level-synchronous traversal
+    if constexpr (kMode == 2) {      // NEXT-3: Alg. 2 level-synchronous traversal
       const Problem PL = kp.chains[c];
       leveled_chain(kp, a, PL, sm, sh);
       continue;
@@ -118,8 +120,8 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
     // instead of pinning 16 registers across the whole traversal
     if (threadIdx.x == 0) sh.prob = kp.chains[c];
     __syncthreads();
-    if constexpr (kMB) chain_worker_mb(kp, sh.prob, sm, sh, sh2, epoch);
-    else chain_worker(kp, sh.prob, sm, sh, epoch);
+    if constexpr (kMode == 1) chain_worker_mb(kp, sh.prob, sm, sh, sh2, epoch);
+    else if constexpr (kMode == 0) chain_worker(kp, sh.prob, sm, sh, epoch);
     grid_barrier(kp);
     chain_reset_signals(kp);
     grid_barrier(kp);
@@ -143,7 +145,7 @@ __device__ __forceinline__ void schedule_phase(const KParams& kp, const MainArgs
 
 // One launch per call: reset -> prologue -> seed / problem set-up ->
 // traversal -> (components -> traversal).  Grid barriers between phases.
-template <int kMinBlocks, bool kMB>
+template <int kMinBlocks, int kMode>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_constant__ KParams kp, const __grid_constant__ MainArgs a) {
   __shared__ ShState sh;
   __shared__ ShState sh2;   // second batch context (multi-batch execution, kMB only)
@@ -189,13 +191,13 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) k_main(const __grid_cons
   grid_barrier(kp);
   stamp(kp, 2);
   // ---- phase 3: the traversal (a2-a12)
-  schedule_phase<kMB>(kp, a, sm, sh, sh2);
+  schedule_phase<kMode>(kp, a, sm, sh, sh2);
   grid_barrier(kp);
   stamp(kp, 3);
   // ---- phase 4: components left over by the chain-first pass (a13)
   if (ld_cg_s32(&kp.ctl->incomplete) && !ld_cg_s32(&kp.ctl->status)) {
     cc_phase(kp, a, sm, sh);
-    schedule_phase<kMB>(kp, a, sm, sh, sh2);
+    schedule_phase<kMode>(kp, a, sm, sh, sh2);
     grid_barrier(kp);
   }
   stamp(kp, 4);
