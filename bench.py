@@ -8,8 +8,10 @@ per-matrix random relabel, MIN_DEGREE start per matrix -- DESIGN.md "Input
 recipe".  A step = one rcm_reorder_batched call (all 8,192 matrices) on
 device-resident input (11 GB, larger than the 126 MB L2); with N > 1 GPUs the
 matrices are sharded (LPT on nnz) and the step includes the NCCL gather of the
-permutations into rank 0.  C4 (R-MAT 2^22, one graph) and C2 (27-point grid
-100^3) are reported in the same line under "secondary" (N = 1 only).
+permutations into rank 0.  C4 (R-MAT 2^22, one graph), C3 (4M-node random
+geometric graph) and C2 (27-point grid 100^3) are reported in the same line
+under "secondary" (N = 1 only), each with the batch chain (default) and the
+level-synchronous schedule (RCM_FLAG_LEVELED) timed side by side.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--config 1..5]
 
@@ -311,6 +313,18 @@ def single_graph(rcm, cfg: int, steps: int, warmup: int, dev, world: int = 1, di
         step()
         perm_h.copy_(perm, non_blocking=True)
     e2e_ms = sum(time_events(e2e_step, steps, stream, flush)) / steps
+    # the same graph through the level-synchronous traversal (NEXT-3, RCM_FLAG_LEVELED)
+    lplan = rcm.Plan(n, nnz, collect_stats=0, flags=rcm.RCM_FLAG_LEVELED)
+    lperm = torch.empty(n, dtype=torch.int32, device=dev)
+
+    def lstep():
+        rcm.rcm_reorder(lplan.handle, n, nnz, rp, ci, mode, start, lperm)
+    for _ in range(max(1, warmup)):
+        lstep()
+    lv_ms = sum(time_events(lstep, steps, stream, flush)) / steps
+    lv_ok = rcm.rcm_sync_status(lplan.handle) == 0
+    lperm_h = lperm.cpu().numpy()
+    lplan.close()
     # start finder (timed apart, as Table I does)
     gl_out = torch.empty(1, dtype=torch.int32, device=dev)
     s0 = int(np.argmax(np.diff(g.row_ptr)))
@@ -350,6 +364,9 @@ def single_graph(rcm, cfg: int, steps: int, warmup: int, dev, world: int = 1, di
         ots.append(time.perf_counter() - t0)
     o_ms = 1e3 * statistics.median(ots)
     res["parity_vs_oracle"] = "bit-identical" if np.array_equal(perm_h.numpy(), ref) else "MISMATCH"
+    res["leveled"] = {"ms": round(lv_ms, 4), "mnodes_per_s": round(n / (lv_ms * 1e-3) / 1e6, 3),
+                      "parity_vs_oracle": "bit-identical" if lv_ok and np.array_equal(lperm_h, ref) else "MISMATCH",
+                      "note": "RCM_FLAG_LEVELED: level-synchronous schedule (Alg. 2), two grid barriers per BFS level"}
     res["start_finder_parity"] = ("identical to oracle.gl" if gl_node == oracle.gl(g.row_ptr, g.col_idx, s0)
                                   else "MISMATCH")
     res["oracle_ms"] = round(o_ms, 3)
@@ -562,7 +579,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=5)
     ap.add_argument("--num-mats", type=int, default=8192)
-    ap.add_argument("--no-secondary", action="store_true", help="skip the C4 / C2 lines (N = 1)")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the C4 / C3 / C2 lines (N = 1)")
     args = ap.parse_args()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         # self-launch N ranks (one process per GPU) on this node
@@ -601,7 +618,7 @@ def main():
         if line is not None:
             line["chain_latency"] = hop
             if world == 1 and not args.no_secondary:
-                line["secondary"] = {f"C{c}": single_graph(rcm, c, 5, 2, dev, hop=hop) for c in (4, 2)}
+                line["secondary"] = {f"C{c}": single_graph(rcm, c, 5, 2, dev, hop=hop) for c in (4, 3, 2)}
     else:
         res = single_graph(rcm, args.config, args.steps, args.warmup, dev, world, dist, hop)
         line = None

@@ -236,6 +236,7 @@ extern "C" rcm_status_t rcm_plan_create(rcm_plan_t* out, int64_t n_max, int64_t 
     }
     p->T = T;
     p->smem = nctx == 1 ? smem_bytes(p->BS, T) : nctx * ((smem_bytes(p->BS, T) + 15) & ~size_t(15));
+    if (o.flags & RCM_FLAG_LEVELED) p->smem = lv_smem_base(p->BS, T) + kLvExtraBytes;   // + staging (rcm_leveled.cuh)
     // one block per SM: the 128-register build (no spills); more: the 64-register build
     p->kernel = pick_kernel(bps, nctx == 2, (o.flags & RCM_FLAG_LEVELED) != 0);
     if (cudaFuncSetAttribute(p->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->smem) != cudaSuccess) {

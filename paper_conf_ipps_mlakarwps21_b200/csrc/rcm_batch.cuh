@@ -112,6 +112,15 @@ __host__ __device__ inline size_t smem_bytes(int BS, int T) {
          sizeof(int32_t) * (size_t)(4 * BS + 2) + 64;
 }
 
+// Leveled traversal (rcm_leveled.cuh): shared memory after the batch layout --
+// the ids of the children the block wrote last, its output buffer, and the
+// long rows of its discovery.
+constexpr int kLvStage = 1024;   // children ids staged per block
+constexpr int kLvOut = 2048;     // children buffered per block before HBM scratch
+constexpr int kLvBig = 512;      // long rows expanded by the whole block (per D pass)
+__host__ __device__ inline size_t lv_smem_base(int BS, int T) { return (smem_bytes(BS, T) + 15) & ~size_t(15); }
+constexpr size_t kLvExtraBytes = 4 * ((size_t)kLvStage + kLvOut + 3 * (size_t)kLvBig + 1);
+
 // Static shared state of one worker.
 constexpr int kLvList = 32;   // leveled traversal: output regions per block and round
 struct ShState {
@@ -132,7 +141,7 @@ struct ShState {
   int64_t spill_base;
   uint32_t* ovbits;            // oversize claims bitmap (shared memory, or HBM scratch for long rows)
   int32_t big_list[256];
-  int32_t lv_off[kLvList], lv_cnt[kLvList], lv_n;   // leveled traversal: this block's output list
+  int32_t lv_off[kLvList], lv_cnt[kLvList], lv_n, lv_outn;   // leveled traversal: this block's output list
   long long clk[10];           // per-stage cycle accumulators (thread 0)
   long long tclk;
   Problem prob;                // the problem being traversed (chain or solo)

@@ -3,38 +3,57 @@
 // permutation as serial RCM and as the batch chain.  It runs inside the
 // persistent kernel; a BFS level costs two grid barriers:
 //
-//   D  discover (Alg. 4 ln 4-9): every node x of the new level
-//      claims its unplaced neighbours n with m_n <- atomicMin(word[n], pos(x)+1)
-//      -- the parent-rank key of the chain (C-4), so after all claims of the
-//      level the owner of n is the earliest parent in o that sees it (Alg. 1
-//      ln 8-12).  Warp-cooperative, load-balanced expansion
-//      (rcm_expand.cuh); rows above kLvBigRow edges are expanded by the block.
+//   D  discover (Alg. 4 ln 4-9): every node x the block just wrote claims its
+//      unplaced neighbours n with m_n <- atomicMin(word[n], pos(x)+1) -- the
+//      parent-rank key of the chain (C-4), so after all claims of the level
+//      the owner of n is the earliest parent in o that sees it (Alg. 1 ln 8-12,
+//      P:L202-212).  Warp-cooperative, load-balanced expansion
+//      (rcm_expand.cuh); rows above kLvWarpRow edges go to one block-wide pass.
 //   == grid barrier (every claim of the level is final: the paper's
 //      "Discovered" for all batches of the level at once)
-//   R  rediscover + sort + count, per batch of <= B_s parents / <= T edge slots
-//      (the chain's load_parents / sort_segments): a child n is kept by parent
-//      p iff owner(n) == pos(p)+1 (Alg. 5 ln 16-17); each parent's children
-//      sorted by (valence, id) (C-1); duplicate entries of a row
-//      collapse after the sort (C-8).  Kept ids go to HBM scratch in order.
+//   R  rediscover + sort + count over an even share of the level, in batches of
+//      <= B_s parents / <= T edge slots (the chain's segments and sort_segments): a
+//      child n is kept by parent p iff owner(n) == pos(p)+1 (Alg. 5 ln 16-17);
+//      each parent's children sorted by (valence, id) (C-1); duplicate
+//      entries of a row collapse after the sort (C-8).  Kept ids are buffered
+//      in shared memory (HBM scratch past kLvOut).
 //   == grid barrier (every block's child count is published)
 //   W  prefix of the block counts (the paper's Counted), output with fused
-//      reverse, then D of the children this block just wrote.
+//      reverse, then D of the children this block wrote (their ids
+//      kept in shared memory; D stores their row starts and valences by
+//      position, so R of the next level loads a parent with one round trip).
 //
-// A level wider than nblocks x B_s parents runs in rounds (R == W per round).
-// If one block's output is far above the mean, the next D is re-balanced
-// over all blocks behind one more barrier.
+// A level wider than nblocks x B_s parents runs in rounds (R..D per round).  If
+// one block's output is far above the mean, that D is spread over all blocks
+// behind one more barrier.
 #pragma once
 #include "rcm_components.cuh"
 
 namespace rcm {
 
 constexpr int kLvU = 4;            // edges per lane in flight (D)
-constexpr int kLvBigRow = 2048;    // rows longer than this are expanded by the whole block (D)
+constexpr int kLvWarpRow = 64;     // rows longer than this are expanded block-wide (D)
+static_assert(kLvBig <= kThreads, "one long row per thread in the block scan");
 
-// D over the nodes at matrix-local positions [x0, x1): claim every neighbour
-// whose owner key is larger than pos + 1.  Block-local work, no barrier.
-static __device__ void lv_discover(const KParams& kp, const Problem& P, ShState& sh, int x0, int x1) {
-  const int cnt = x1 - x0;
+__device__ __forceinline__ int32_t* lv_sm(const KParams& kp) {
+  return reinterpret_cast<int32_t*>(rcm_dsm + lv_smem_base(kp.BS, kp.T));
+}
+__device__ __forceinline__ int32_t* lv_st_v(const KParams& kp) { return lv_sm(kp); }
+__device__ __forceinline__ int32_t* lv_out(const KParams& kp) { return lv_sm(kp) + kLvStage; }
+__device__ __forceinline__ int32_t* lv_bg_rs(const KParams& kp) { return lv_out(kp) + kLvOut; }
+__device__ __forceinline__ int32_t* lv_bg_key(const KParams& kp) { return lv_bg_rs(kp) + kLvBig; }
+__device__ __forceinline__ int32_t* lv_bg_pre(const KParams& kp) { return lv_bg_key(kp) + kLvBig; }   // kLvBig + 1
+
+__device__ __forceinline__ void lv_claim(unsigned long long* word, int c, unsigned long long wv, uint32_t k) {
+  if (c >= 0 && (uint32_t)(wv >> 32) > k) atomicMin(word + c, ((unsigned long long)k << 32) | (wv & 0xffffffffull));
+}
+
+// D over the nodes at matrix-local positions [x0, x0 + cnt): claim every
+// neighbour whose owner key is larger than pos + 1.  `staged`: the ids are in
+// lv_st_v (written by W), else in o[].  Row starts / valences are stored by
+// position (prs, pdeg) for R.  Block-local work, no barrier.
+static __device__ void lv_discover(const KParams& kp, const Problem& P, const CompWS& w, ShState& sh, int x0, int cnt,
+                                   bool staged) {
   if (cnt <= 0) return;   // block-uniform
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int32_t* o = kp.o + P.o_base;
@@ -49,13 +68,16 @@ static __device__ void lv_discover(const KParams& kp, const Problem& P, ShState&
     int rs = 0, d = 0;
     uint32_t key = 0;
     if (lane < per && i < cnt) {
-      const int v = ld_cg_s32(o + x0 + i);
+      const int v = staged ? lv_st_v(kp)[i] : ld_cg_s32(o + x0 + i);
       rs = __ldg(rp + v);
       d = __ldg(rp + v + 1) - rs;
       key = (uint32_t)(x0 + i) + 1u;
-      if (d > kLvBigRow) {
+      w.front0[P.o_base + x0 + i] = rs;   // prs
+      w.front1[P.o_base + x0 + i] = d;    // pdeg
+      if (d > kLvWarpRow) {
         const int k = atomicAdd(&sh.big_n, 1);
-        if (k < 256) { sh.big_list[k] = i; d = 0; }   // else: expanded here by the warp
+        if (k < kLvBig) { lv_bg_rs(kp)[k] = rs; lv_bg_key(kp)[k] = (int)key; lv_bg_pre(kp)[k] = d; d = 0; }
+        // else: expanded here by the warp
       }
     }
     WarpRows R;
@@ -67,35 +89,41 @@ static __device__ void lv_discover(const KParams& kp, const Problem& P, ShState&
 #pragma unroll
       for (int u = 0; u < kLvU; ++u) wv[u] = c[u] >= 0 ? ld_weak_u64(word + c[u]) : 0ull;   // prefilter
 #pragma unroll
-      for (int u = 0; u < kLvU; ++u) {
-        const uint32_t k = __shfl_sync(kFull, key, j[u] & 31);
-        if (c[u] >= 0 && (uint32_t)(wv[u] >> 32) > k)
-          atomicMin(word + c[u], ((unsigned long long)k << 32) | (wv[u] & 0xffffffffull));
-      }
+      for (int u = 0; u < kLvU; ++u) lv_claim(word, c[u], wv[u], __shfl_sync(kFull, key, j[u] & 31));
     }
   }
   __syncthreads();
-  const int nbig = min(sh.big_n, 256);
-  for (int bi = 0; bi < nbig; ++bi) {   // long rows: the whole block, kLvU edges per thread in flight
-    const int i = sh.big_list[bi];
-    const int v = ld_cg_s32(o + x0 + i);
-    const int rs = __ldg(rp + v), re = __ldg(rp + v + 1);
-    const uint32_t k = (uint32_t)(x0 + i) + 1u;
-    for (int e0 = rs + threadIdx.x; e0 < re; e0 += kThreads * kLvU) {
-      int c[kLvU];
-      unsigned long long wv[kLvU];
+  const int nbig = min(sh.big_n, kLvBig);
+  if (nbig == 0) return;
+  // long rows: one block-wide flattened pass over all of them
+  int tot;
+  const int len = threadIdx.x < nbig ? lv_bg_pre(kp)[threadIdx.x] : 0;
+  const int ex = block_exclusive_scan<int32_t>(len, sh.wtmp32, tot);
+  if (threadIdx.x < nbig) lv_bg_pre(kp)[threadIdx.x] = ex;
+  if (threadIdx.x == 0) lv_bg_pre(kp)[nbig] = tot;
+  __syncthreads();
+  for (int e0 = threadIdx.x; e0 < tot; e0 += kThreads * kLvU) {
+    int c[kLvU], jj[kLvU];
 #pragma unroll
-      for (int u = 0; u < kLvU; ++u) {
-        const int e = e0 + u * kThreads;
-        c[u] = e < re ? __ldg(col + e) : -1;
+    for (int u = 0; u < kLvU; ++u) {
+      const int e = e0 + u * kThreads;
+      c[u] = -1;
+      jj[u] = 0;
+      if (e < tot) {
+        int lo = 0, hi = nbig - 1;   // last row with pre <= e
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (lv_bg_pre(kp)[mid] <= e) lo = mid; else hi = mid - 1;
+        }
+        jj[u] = lo;
+        c[u] = __ldg(col + lv_bg_rs(kp)[lo] + (e - lv_bg_pre(kp)[lo]));
       }
-#pragma unroll
-      for (int u = 0; u < kLvU; ++u) wv[u] = c[u] >= 0 ? ld_weak_u64(word + c[u]) : 0ull;
-#pragma unroll
-      for (int u = 0; u < kLvU; ++u)
-        if (c[u] >= 0 && (uint32_t)(wv[u] >> 32) > k)
-          atomicMin(word + c[u], ((unsigned long long)k << 32) | (wv[u] & 0xffffffffull));
     }
+    unsigned long long wv[kLvU];
+#pragma unroll
+    for (int u = 0; u < kLvU; ++u) wv[u] = c[u] >= 0 ? ld_weak_u64(word + c[u]) : 0ull;
+#pragma unroll
+    for (int u = 0; u < kLvU; ++u) lv_claim(word, c[u], wv[u], c[u] >= 0 ? (uint32_t)lv_bg_key(kp)[jj[u]] : 0u);
   }
   __syncthreads();
 }
@@ -124,7 +152,8 @@ static __device__ void lv_list_push(const KParams& kp, const CompWS& w, ShState&
       }
     }
     __syncthreads();
-    if (threadIdx.x == 0) { sh.lv_off[0] = nb; sh.lv_cnt[0] = tot; sh.lv_n = 1; }
+    // on a capacity error (latched) the list is dropped: no read past the scratch
+    if (threadIdx.x == 0) { sh.lv_off[0] = max(nb, 0); sh.lv_cnt[0] = nb >= 0 ? tot : 0; sh.lv_n = 1; }
     __syncthreads();
   }
   if (threadIdx.x == 0) { sh.lv_off[sh.lv_n] = base; sh.lv_cnt[sh.lv_n] = cnt; ++sh.lv_n; }
@@ -132,7 +161,9 @@ static __device__ void lv_list_push(const KParams& kp, const CompWS& w, ShState&
 }
 
 // The sorted, kept children of a batch (segments cand[p_eo[lp] .. + p_cnt[lp]))
-// -> HBM scratch in slot order, duplicates (adjacent after the sort) dropped.
+// in slot order, duplicates (adjacent after the sort) dropped: appended to the
+// block's shared-memory output buffer while it fits and no HBM entry exists
+// yet, else to HBM scratch as the next entry of the block's list.
 static __device__ void lv_emit(const KParams& kp, const CompWS& w, ShState& sh, int32_t* gcur, int E) {
   const int per = (E + kThreads - 1) / kThreads;
   const int b0 = min(E, threadIdx.x * per), b1 = min(E, b0 + per);
@@ -147,9 +178,19 @@ static __device__ void lv_emit(const KParams& kp, const CompWS& w, ShState& sh, 
   int tot;
   int r = block_exclusive_scan<int32_t>(k, sh.wtmp32, tot);
   if (tot == 0) return;
-  if (threadIdx.x == 0) sh.k = lv_alloc(kp, w, gcur, tot);
+  const int outn = sh.lv_outn;   // ids in the shared buffer (thread 0 updates it below, after the reads)
+  if (sh.lv_n == 0 && outn + tot <= kLvOut) {
+    for (int e = b0; e < b1; ++e)
+      if (valid(e)) lv_out(kp)[outn + r++] = (int)(uint32_t)cand[e];
+    __syncthreads();
+    if (threadIdx.x == 0) sh.lv_outn = outn + tot;
+    __syncthreads();
+    return;
+  }
   __syncthreads();
-  const int base = sh.k;
+  if (threadIdx.x == 0) sh.count = lv_alloc(kp, w, gcur, tot);
+  __syncthreads();
+  const int base = sh.count;
   if (base >= 0)
     for (int e = b0; e < b1; ++e)
       if (valid(e)) w.vals1[base + r++] = (int)(uint32_t)cand[e];
@@ -217,17 +258,59 @@ static __device__ void lv_oversize(const KParams& kp, const Problem& P, const Co
   if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
 }
 
-// R over this block's parents [cb, ce) of the current level: batches of
-// <= Bg parents / <= T edge slots, each rediscovered, sorted and emitted.
-static __device__ void lv_rediscover(const KParams& kp, const Problem& P, const CompWS& w, const SmemPtrs& sm,
-                                     ShState& sh, int32_t* gcur, int32_t* scur, int cb, int ce) {
+// load_parents (rcm_batch.cuh) for the parents at positions [q0, q0 + nP):
+// id, row start and valence in one round trip (o[], and prs / pdeg written by
+// D).  Cuts at T edge slots; sh.E = slots.
+static __device__ int lv_parents(const KParams& kp, const Problem& P, const CompWS& w, ShState& sh, int q0, int nP) {
+  for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
+    const int64_t x = P.o_base + q0 + lp;
+    sm_p_v(kp)[lp] = ld_cg_s32(kp.o + x);
+    sm_p_rs(kp)[lp] = ld_cg_s32(w.front0 + x);
+    sm_p_eo(kp)[lp] = ld_cg_s32(w.front1 + x);
+  }
+  __syncthreads();
+  int E = block_scan_array<int32_t>(sm_p_eo(kp), nP, sh.wtmp32);
+  sm_p_eo(kp)[nP] = E;
+  __syncthreads();
+  if (E > kp.T && nP > 1) {   // longest prefix whose edges fit T (at least one parent)
+    if (threadIdx.x == 0) {
+      int lo = 1, hi = nP;
+      while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (sm_p_eo(kp)[mid] <= kp.T) lo = mid; else hi = mid - 1;
+      }
+      sh.nP = lo;
+    }
+    __syncthreads();
+    nP = sh.nP;
+    E = sm_p_eo(kp)[nP];
+  }
+  if (threadIdx.x == 0) { sh.nP = nP; sh.E = E; }
+  if (E <= kp.T) {
+    const int lane = threadIdx.x & 31;
+    for (int lp = threadIdx.x >> 5; lp < nP; lp += kWarps) {
+      const int eb = sm_p_eo(kp)[lp], ee = sm_p_eo(kp)[lp + 1];
+      for (int j = eb + lane; j < ee; j += 32) sm_lpof(kp)[j] = (uint16_t)lp;
+    }
+  }
+  __syncthreads();
+  return nP;
+}
+
+// R over the parents at positions [x0, x0 + cnt): batches of <= Bg parents /
+// <= T edge slots, each rediscovered, sorted and emitted.  Returns the block's
+// child count.
+static __device__ int lv_rediscover(const KParams& kp, const Problem& P, const CompWS& w, const SmemPtrs& sm,
+                                    ShState& sh, int32_t* gcur, int32_t* scur, int x0, int cnt) {
   const int32_t* col = kp.col_idx + P.ci_base;
   const unsigned long long* word = kp.word + P.node_base;
-  for (int ob = cb; ob < ce;) {
-    const int nP = load_parents(kp, P, sm, sh, ob, min(kp.Bg, ce - ob), true);
+  if (threadIdx.x == 0) { sh.lv_n = 0; sh.lv_outn = 0; }
+  __syncthreads();
+  for (int ob = 0; ob < cnt;) {
+    const int nP = lv_parents(kp, P, w, sh, x0 + ob, min(kp.Bg, cnt - ob));
     const int E = sh.E;
     if (E > kp.T) {   // nP == 1, oversize
-      lv_oversize(kp, P, w, sh, gcur, scur, ob);
+      lv_oversize(kp, P, w, sh, gcur, scur, x0 + ob);
       ob += 1;
       __syncthreads();
       continue;
@@ -235,7 +318,7 @@ static __device__ void lv_rediscover(const KParams& kp, const Problem& P, const 
     for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm_p_cnt(kp)[lp] = 0;
     __syncthreads();
     // rediscovery (Alg. 5 ln 16-17): keep n iff owner(n) == key(p)
-    const uint32_t kfirst = (uint32_t)ob + 1u;
+    const uint32_t kfirst = (uint32_t)(x0 + ob) + 1u;
     for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
       int c[kDiscU];
 #pragma unroll
@@ -267,6 +350,9 @@ static __device__ void lv_rediscover(const KParams& kp, const Problem& P, const 
     ob += nP;
     __syncthreads();
   }
+  int myc = sh.lv_outn;
+  for (int j = 0; j < sh.lv_n; ++j) myc += sh.lv_cnt[j];
+  return myc;
 }
 
 static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const Problem& P, const SmemPtrs& sm,
@@ -283,34 +369,32 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
     gcur[0] = gcur[1] = scur[0] = scur[1] = 0;
     stat_add(kp, &kp.stats->components, 1);
   }
+  if (b == 0 && threadIdx.x == 0) lv_st_v(kp)[0] = P.seed;
+  __syncthreads();
+  lv_discover(kp, P, w, sh, P.pos0, b == 0 ? 1 : 0, true);
   grid_barrier(kp);
-  if (b == 0) lv_discover(kp, P, sh, P.pos0, P.pos0 + 1);
-  grid_barrier(kp);
-  int lb = P.pos0, le = P.pos0 + 1, par = 0;
-  const int per_round = nb * kp.Bg;
   // per-round timeline of block 0 (collect_stats == 3): R start, R end, after
-  // barrier 1, output written, D done, after the level barrier; children, level
+  // barrier 1, output written, D done, after the level barrier; children,
+  // level, max block output
   int nround = (b == 0 && threadIdx.x == 0) ? (int)kp.ctl->dbg[6] : 0;   // across the problems of a call
   auto tr = [&](int k, unsigned long long v) {
     if (kp.trace && b == 0 && threadIdx.x == 0 && nround < kp.trace_cap) kp.trace[(size_t)nround * kTraceW + k] = v;
   };
+  int lb = P.pos0, le = P.pos0 + 1, par = 0;
+  const int per_round = nb * kp.Bg;
   for (int level = 0;; ++level) {
     int32_t* gc = gcur + (level & 1);
     int32_t* sc = scur + (level & 1);
     int le_next = le;
     for (int rb = lb; rb < le; rb += per_round) {
-      // ---- R: this block's share of the round
+      // ---- R: an even share of the round
       const int re_ = min(le, rb + per_round);
       const int m = (re_ - rb + nb - 1) / nb;
       const int cb = min(re_, rb + b * m), ce = min(re_, cb + m);
-      if (threadIdx.x == 0) sh.lv_n = 0;
-      __syncthreads();
       tr(0, globaltimer());
-      lv_rediscover(kp, P, w, sm, sh, gc, sc, cb, ce);
-      tr(1, globaltimer());
-      int myc = 0;
-      for (int j = 0; j < sh.lv_n; ++j) myc += sh.lv_cnt[j];
+      const int myc = lv_rediscover(kp, P, w, sm, sh, gc, sc, cb, ce - cb);
       if (threadIdx.x == 0) st_relaxed_s32(btot + par * kMaxBlocks + b, myc);
+      tr(1, globaltimer());
       grid_barrier(kp);
       tr(2, globaltimer());
       // ---- W: prefix of the block counts, output with fused reverse
@@ -330,31 +414,33 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       __syncthreads();
       long long maxc = 0;
       for (int i = 0; i < kWarps; ++i) maxc = max(maxc, sh.wtmp64b[i]);
-      const int x0 = le_next + sh.written;
-      // flattened copy of the block's list: position x0 + i
-      int run = 0;
+      const int xw = le_next + sh.written;
+      auto put = [&](int i, int c) {
+        const int x = xw + i;
+        o[x] = c;
+        perm[P.mat_n - 1 - x] = c;
+        if (kp.iperm) kp.iperm[P.node_base + c] = P.mat_n - 1 - x;
+        if (i < kLvStage) lv_st_v(kp)[i] = c;
+      };
+      const int outn = sh.lv_outn;
+      for (int i = threadIdx.x; i < outn; i += kThreads) put(i, lv_out(kp)[i]);
+      int run = outn;
       for (int j = 0; j < sh.lv_n; ++j) {
-        const int off = sh.lv_off[j], cnt = sh.lv_cnt[j];
-        for (int i = threadIdx.x; i < cnt; i += kThreads) {
-          const int c = __ldcg(w.vals1 + off + i);
-          const int x = x0 + run + i;
-          o[x] = c;
-          perm[P.mat_n - 1 - x] = c;
-          if (kp.iperm) kp.iperm[P.node_base + c] = P.mat_n - 1 - x;
-        }
-        run += cnt;
+        const int off = sh.lv_off[j], n = sh.lv_cnt[j];
+        for (int i = threadIdx.x; i < n; i += kThreads) put(run + i, __ldcg(w.vals1 + off + i));
+        run += n;
       }
       __syncthreads();
       tr(3, globaltimer());
       // ---- D of the next level
       const long long mean = (total + nb - 1) / nb;
       if (maxc <= 4 * mean + 256) {
-        lv_discover(kp, P, sh, x0, x0 + myc);     // the children this block wrote
-      } else {                                      // skewed: spread the claims over all blocks
+        lv_discover(kp, P, w, sh, xw, myc, myc <= kLvStage);   // the children this block wrote
+      } else {                                                  // skewed: spread over all blocks
         grid_barrier(kp);
-        const int mm = (total + nb - 1) / nb;
+        const int mm = (int)mean;
         const int d0 = min(total, b * mm), d1 = min(total, d0 + mm);
-        lv_discover(kp, P, sh, le_next + d0, le_next + d1);
+        lv_discover(kp, P, w, sh, le_next + d0, d1 - d0, false);
       }
       tr(4, globaltimer());
       tr(8, (unsigned long long)total);

@@ -1,5 +1,5 @@
 """Per-round timeline of the leveled traversal (RCM_FLAG_LEVELED, collect_stats=3),
-block 0's view: R, barrier 1, W (prefix + output), D, level barrier (us).
+block 0's view per round: R, barrier 1, W (prefix + output), D, level barrier (us).
 usage: python tools/trace_leveled.py <cfg> [opts-dict]"""
 import ctypes, json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
