@@ -117,7 +117,7 @@ __host__ __device__ inline size_t smem_bytes(int BS, int T) {
 // long rows of its discovery.
 constexpr int kLvStage = 1024;   // children ids staged per block
 constexpr int kLvOut = 2048;     // children buffered per block before HBM scratch
-constexpr int kLvBig = 512;      // long rows expanded by the whole block (per D pass)
+constexpr int kLvBig = 256;      // long rows expanded by the whole block (per D pass)
 __host__ __device__ inline size_t lv_smem_base(int BS, int T) { return (smem_bytes(BS, T) + 15) & ~size_t(15); }
 constexpr size_t kLvExtraBytes = 4 * ((size_t)kLvStage + kLvOut + 3 * (size_t)kLvBig + 1);
 

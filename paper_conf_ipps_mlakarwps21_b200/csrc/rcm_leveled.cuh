@@ -397,6 +397,7 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       tr(1, globaltimer());
       grid_barrier(kp);
       tr(2, globaltimer());
+      tr(6, (unsigned long long)kp.ctl->dbg[7]);
       // ---- W: prefix of the block counts, output with fused reverse
       if (gtid() == 0) { gcur[(level + 1) & 1] = 0; scur[(level + 1) & 1] = 0; }
       int total = 0, mx = 0;
@@ -451,7 +452,7 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       ++nround;
     }
     grid_barrier(kp);
-    if (nround > 0) { --nround; tr(5, globaltimer()); ++nround; }
+    if (nround > 0) { --nround; tr(5, globaltimer()); tr(7, (unsigned long long)kp.ctl->dbg[7]); ++nround; }
     if (le_next == le) break;
     lb = le;
     le = le_next;

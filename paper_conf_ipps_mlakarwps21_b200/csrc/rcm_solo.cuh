@@ -248,6 +248,13 @@ __device__ __forceinline__ void so_set(const SoloMat& M, uint32_t* bits, int v) 
   v += M.b0;
   atomicOr(bits + (v >> 5), 1u << (v & 31));
 }
+// placed-bit set on the hot path: the shared-memory bitmap addressed as shared
+// (ATOMS) for small matrices, the HBM bitmap otherwise
+template <bool kBig>
+__device__ __forceinline__ void so_place(const SoloMat& M, int v) {
+  if constexpr (kBig) so_set(M, M.vis, v);
+  else atomicOr(reinterpret_cast<uint32_t*>(so_base() + kSoOffVis) + (v >> 5), 1u << (v & 31));
+}
 // test-and-set, true if this call set the bit
 __device__ __forceinline__ bool so_claim_bit(const SoloMat& M, uint32_t* bits, int v) {
   v += M.b0;
@@ -565,15 +572,16 @@ __device__ __forceinline__ int so_scan1(int v, int32_t* buf, int& total) {
   }
   if (lane == 31) buf[wid] = x;
   __syncthreads();
-  int base = 0, tot = 0;
+  // the kSoloNW warp totals, scanned in the first lanes of every warp
+  int wv = lane < kSoloNW ? buf[lane] : 0;
 #pragma unroll
-  for (int w = 0; w < kSoloNW; ++w) {
-    const int t = buf[w];
-    base += w < wid ? t : 0;
-    tot += t;
+  for (int d = 1; d < kSoloNW; d <<= 1) {
+    const int y = __shfl_up_sync(0xffffffffu, wv, d);
+    if (lane >= d) wv += y;
   }
-  total = tot;
-  return base + x - v;
+  total = __shfl_sync(0xffffffffu, wv, kSoloNW - 1);
+  const int base = __shfl_sync(0xffffffffu, wv, (wid + 31) & 31);   // inclusive total of warps < wid
+  return (wid ? base : 0) + x - v;
 }
 
 // Traversal state, block-uniform, held in registers by every thread.
@@ -613,7 +621,7 @@ static __device__ void so_oversize(const SoloArgs& a, const SoloMat& M, SoloSh& 
       if (ins[u]) {   // one parent: every child is kept, once (duplicates share the entry)
         const int idx = atomicAdd(&sh.cnt, 1);
         keys[idx] = ((unsigned long long)(uint32_t)(cre[u] - crs[u]) << 32) | (uint32_t)cc[u];
-        so_set(M, M.vis, cc[u]);
+        so_place<kBig>(M, cc[u]);
         so_unclaim<kBig>(slot[u]);
       }
     }
@@ -692,18 +700,24 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
   // ---- discover: columns, placed test, claims; first claimers load the child's row_ptr
   const int e0 = t * kSoloU;
   int cc[kSoloU], slot[kSoloU];   // slot >= 0: this thread created the child's table entry
-  {
-    int lp = e0 < E ? so_flp()[t] : 0;
+  if (e0 < E) {
+    // the parent of the thread's first slot, then advance: its row start and
+    // slot range stay in registers across the kSoloU slots
+    int lp = so_flp()[t];
+    int se = so_p_eo()[lp], nx = so_p_eo()[lp + 1], rs = so_p_rs()[lp];
 #pragma unroll
     for (int u = 0; u < kSoloU; ++u) {
       const int e = e0 + u;
       cc[u] = -1;
       if (e < E) {
-        while (so_p_eo()[lp + 1] <= e) ++lp;
+        while (nx <= e) { ++lp; se = nx; nx = so_p_eo()[lp + 1]; rs = so_p_rs()[lp]; }
         so_lpof()[e] = (uint16_t)lp;
-        cc[u] = SO_LD(M.col + so_p_rs()[lp] + (e - so_p_eo()[lp]));
+        cc[u] = SO_LD(M.col + rs + (e - se));
       }
     }
+  } else {
+#pragma unroll
+    for (int u = 0; u < kSoloU; ++u) cc[u] = -1;
   }
 #pragma unroll
   for (int u = 0; u < kSoloU; ++u) {
@@ -736,7 +750,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
       if constexpr (!kBig) key = (dg << 32) | ((unsigned long long)(uint32_t)c << 15) | (uint32_t)sl;
       else key = (dg << 32) | (uint32_t)c;
       so_cand()[so_p_eo()[lp] + idx] = key;
-      so_set(M, M.vis, c);
+      so_place<kBig>(M, c);
       so_unclaim<kBig>(sl);   // each entry is read by its creator only
       ++won;
     }

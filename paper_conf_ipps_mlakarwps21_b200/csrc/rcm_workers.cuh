@@ -26,19 +26,24 @@ static __device__ void grid_barrier(const KParams& kp) {
   beacon(kp, 11, -1, ld_relaxed_s32(&kp.ctl->gbar_gen));
   __syncthreads();
   if (threadIdx.x == 0) {
-    int gen = ld_acquire_s32(&kp.ctl->gbar_gen);
-    __threadfence();
-    int arrived = atomicAdd(&kp.ctl->gbar_count, 1);
+    // the generation this barrier ends: a relaxed read cannot return an older
+    // value than the one this thread observed at the previous barrier, and the
+    // count cannot complete without this block
+    const int gen = ld_relaxed_s32(&kp.ctl->gbar_gen);
+    int arrived;   // acq_rel: releases this block's writes (after bar.sync), acquires the earlier arrivals
+    asm volatile("atom.add.acq_rel.gpu.global.s32 %0, [%1], 1;" : "=r"(arrived) : "l"(&kp.ctl->gbar_count) : "memory");
     if (arrived == kp.nblocks - 1) {
-      atomicExch(&kp.ctl->gbar_count, 0);
-      __threadfence();
+      if (kp.trace) kp.ctl->dbg[7] = (long long)globaltimer();   // last arrival (leveled trace)
+      st_relaxed_s32(&kp.ctl->gbar_count, 0);
       st_release_s32(&kp.ctl->gbar_gen, gen + 1);
     } else {
+      // relaxed polling + one acquire fence (an ld.acquire per poll would drop the SM's L1 each time)
       uint64_t t0 = globaltimer();
-      while (ld_acquire_s32(&kp.ctl->gbar_gen) == gen) {
-        __nanosleep(64);
+      while (ld_relaxed_s32(&kp.ctl->gbar_gen) == gen) {
+        __nanosleep(32);
         if (globaltimer() - t0 > kWatchdogNs) { latch_hang(kp.ctl, 4, gen, 0, 0); break; }
       }
+      fence_acquire_gpu();
     }
   }
   __syncthreads();

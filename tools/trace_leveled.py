@@ -26,6 +26,12 @@ nxt = np.append(tr[1:, 0], tr[-1, 4])
 end = np.where(tr[:, 5] > 0, tr[:, 5], nxt)
 ph = {"R": tr[:, 1] - tr[:, 0], "bar1": tr[:, 2] - tr[:, 1], "W": tr[:, 3] - tr[:, 2], "D": tr[:, 4] - tr[:, 3],
       "bar2": end - tr[:, 4]}
+# barrier split (rows with a level barrier): wait for the last block vs release latency
+lvl = tr[:, 5] > 0
+ph["b1_wait_last"] = tr[:, 6] - tr[:, 1]
+ph["b1_release"] = tr[:, 2] - tr[:, 6]
+ph["b2_wait_last"] = np.where(lvl, tr[:, 7] - tr[:, 4], 0)
+ph["b2_release"] = np.where(lvl, tr[:, 5] - tr[:, 7], 0)
 tot = {k: round(float(v.sum()) / 1000, 1) for k, v in ph.items()}
 print(json.dumps({"cfg": cfg, "rounds": len(tr), "levels": int(tr[:, 9].max()) + 1 if len(tr) else 0,
                   "span_us": round(float(end[-1] - tr[0, 0]) / 1000, 1), "sum_us": tot,
