@@ -233,8 +233,29 @@ def test_hub_above_the_claims_bitmap(rcm):
     has no valence limit)."""
     g = synth.relabel(synth.star(700000), synth.randperm(700001, 9))
     ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.MIN_DEGREE)
-    for path in ("default", "chain", "serial"):
+    for path in ("default", "chain", "serial", "leveled"):
         assert np.array_equal(_run(rcm, g, oracle.MIN_DEGREE, 0, **PATHS[path]), ref), path
+
+
+def test_leveled_wide_levels_and_overflow(rcm):
+    """Leveled schedule (NEXT-3) under stress: a level of 5,920 parents of
+    valence ~1,200 > T/2 (one batch each: 40 batches per block and round, so
+    the block's output list is merged), rounds (level wider than blocks x B_s),
+    a skewed output (every grandchild written by few blocks is re-spread), per
+    block outputs above the shared-memory buffer (HBM scratch), long rows in the
+    block-wide discovery pass, duplicate entries (test-side mutator)."""
+    rng = np.random.default_rng(21)
+    P, deg, G = 5920, 1200, 400_000
+    par = np.repeat(np.arange(1, P + 1), deg)
+    gc = 1 + P + rng.integers(0, G, P * deg)
+    src = np.concatenate([np.zeros(P, np.int64), par])
+    dst = np.concatenate([np.arange(1, P + 1), gc])
+    g = synth.csr_from_pairs(1 + P + G, src, dst)
+    g = mutate.mutate(g, 22, dup=0.01)
+    ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.FIXED, 0)
+    opts = dict(flags=8 | 32, solo_threshold=-1, blocks_per_sm=1, temp_elems=2304, batch_nodes=64)
+    assert np.array_equal(_run(rcm, g, oracle.FIXED, 0, **opts), ref)
+    assert np.array_equal(_run(rcm, g, oracle.FIXED, 0, **PATHS["leveled"]), ref)
 
 
 def test_batched_matrices_above_the_shared_bitmap(rcm):
