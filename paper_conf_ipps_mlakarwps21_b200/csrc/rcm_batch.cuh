@@ -141,7 +141,7 @@ struct ShState {
   int64_t spill_base;
   uint32_t* ovbits;            // oversize claims bitmap (shared memory, or HBM scratch for long rows)
   int32_t big_list[256];
-  int32_t lv_off[kLvList], lv_cnt[kLvList], lv_n, lv_outn;   // leveled traversal: this block's output list
+  int32_t lv_off[kLvList], lv_cnt[kLvList], lv_n, lv_outn, lv_cap;   // leveled traversal: this block's output list
   long long clk[10];           // per-stage cycle accumulators (thread 0)
   long long tclk;
   Problem prob;                // the problem being traversed (chain or solo)

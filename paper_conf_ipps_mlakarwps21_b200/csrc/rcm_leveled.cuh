@@ -128,36 +128,37 @@ static __device__ void lv_discover(const KParams& kp, const Problem& P, const Co
   __syncthreads();
 }
 
-// Append `cnt` ids (already in order) as the next entry of this block's output
-// list; when the list is full its entries are first merged into one region.
-__device__ __forceinline__ int lv_alloc(const KParams& kp, const CompWS& w, int32_t* gcur, int cnt) {
-  const int base = atomicAdd(gcur, cnt);
-  if ((long long)base + cnt > w.cap) { latch_error(kp.ctl, ST_CAPACITY); return -1; }
+// HBM scratch for output past the shared buffer: w.ckey viewed as 2n ints
+// (idle during a traversal), cursor per level parity.  A block reserves it in
+// chunks that double with its overflow so far (>= 1,024 ids) and appends
+// consecutive emits to its last chunk: a block's overflow is a few regions,
+// and the level's reservations stay within 2n.
+__device__ __forceinline__ int32_t* lv_ovf(const CompWS& w) { return reinterpret_cast<int32_t*>(w.ckey); }
+__device__ __forceinline__ int lv_alloc(const KParams& kp, long long cap, int32_t* cur, int cnt) {
+  const int base = atomicAdd(cur, cnt);
+  if ((long long)base + cnt > cap) { latch_error(kp.ctl, ST_CAPACITY); return -1; }
   return base;
 }
-static __device__ void lv_list_push(const KParams& kp, const CompWS& w, ShState& sh, int32_t* gcur, int base, int cnt) {
-  // called by all threads; sh.lv_* updated by thread 0
-  if (sh.lv_n == kLvList) {   // merge the list into one contiguous region
-    int tot = 0;
-    for (int j = 0; j < kLvList; ++j) tot += sh.lv_cnt[j];
-    __syncthreads();
-    if (threadIdx.x == 0) sh.k = lv_alloc(kp, w, gcur, tot);
-    __syncthreads();
-    const int nb = sh.k;
-    if (nb >= 0) {
-      int run = 0;
-      for (int j = 0; j < kLvList; ++j) {
-        for (int i = threadIdx.x; i < sh.lv_cnt[j]; i += kThreads) w.vals1[nb + run + i] = __ldcg(w.vals1 + sh.lv_off[j] + i);
-        run += sh.lv_cnt[j];
-      }
-    }
-    __syncthreads();
-    // on a capacity error (latched) the list is dropped: no read past the scratch
-    if (threadIdx.x == 0) { sh.lv_off[0] = max(nb, 0); sh.lv_cnt[0] = nb >= 0 ? tot : 0; sh.lv_n = 1; }
-    __syncthreads();
+// Thread 0: room for `cnt` more overflow ids of this block; returns the write
+// offset in lv_ovf (or -1 on a latched capacity error).  The last entry is
+// extended or a new one opened; the caller writes the ids.
+__device__ __forceinline__ int lv_ovf_reserve(const KParams& kp, const CompWS& w, ShState& sh, int32_t* gcur, int cnt) {
+  if (sh.lv_n > 0 && sh.lv_cnt[sh.lv_n - 1] + cnt <= sh.lv_cap) {
+    const int at = sh.lv_off[sh.lv_n - 1] + sh.lv_cnt[sh.lv_n - 1];
+    sh.lv_cnt[sh.lv_n - 1] += cnt;
+    return at;
   }
-  if (threadIdx.x == 0) { sh.lv_off[sh.lv_n] = base; sh.lv_cnt[sh.lv_n] = cnt; ++sh.lv_n; }
-  __syncthreads();
+  if (sh.lv_n == kLvList) { latch_error(kp.ctl, ST_CAPACITY); return -1; }
+  int so_far = 0;
+  for (int j = 0; j < sh.lv_n; ++j) so_far += sh.lv_cnt[j];
+  const int chunk = max(cnt, max(1024, so_far));
+  const int base = lv_alloc(kp, 2 * w.cap, gcur, chunk);
+  if (base < 0) return -1;
+  sh.lv_off[sh.lv_n] = base;
+  sh.lv_cnt[sh.lv_n] = cnt;
+  sh.lv_cap = chunk;
+  ++sh.lv_n;
+  return base;
 }
 
 // The sorted, kept children of a batch (segments cand[p_eo[lp] .. + p_cnt[lp]))
@@ -188,13 +189,13 @@ static __device__ void lv_emit(const KParams& kp, const CompWS& w, ShState& sh, 
     return;
   }
   __syncthreads();
-  if (threadIdx.x == 0) sh.count = lv_alloc(kp, w, gcur, tot);
+  if (threadIdx.x == 0) sh.count = lv_ovf_reserve(kp, w, sh, gcur, tot);
   __syncthreads();
   const int base = sh.count;
   if (base >= 0)
     for (int e = b0; e < b1; ++e)
-      if (valid(e)) w.vals1[base + r++] = (int)(uint32_t)cand[e];
-  lv_list_push(kp, w, sh, gcur, base < 0 ? 0 : base, base < 0 ? 0 : tot);
+      if (valid(e)) lv_ovf(w)[base + r++] = (int)(uint32_t)cand[e];
+  __syncthreads();
 }
 
 // A parent with more than T edges: its kept children counted,
@@ -240,7 +241,7 @@ static __device__ void lv_oversize(const KParams& kp, const Problem& P, const Co
   int u = 0;
   for (int i = threadIdx.x; i < K; i += kThreads) u += i == 0 || key_at(i) != key_at(i - 1);
   const int U = block_reduce_sum<int32_t>(u, sh.wtmp32);
-  if (threadIdx.x == 0) sh.k = lv_alloc(kp, w, gcur, U);
+  if (threadIdx.x == 0) sh.k = lv_ovf_reserve(kp, w, sh, gcur, U);
   __syncthreads();
   const int base = sh.k;
   if (base < 0) return;
@@ -251,10 +252,10 @@ static __device__ void lv_oversize(const KParams& kp, const Problem& P, const Co
     const bool ok = i < K && (i == 0 || x != key_at(i - 1));
     int tot;
     const int r = block_exclusive_scan<int32_t>(ok ? 1 : 0, sh.wtmp32, tot);
-    if (ok) w.vals1[base + run + r] = (int)(uint32_t)x;
+    if (ok) lv_ovf(w)[base + run + r] = (int)(uint32_t)x;
     run += tot;
   }
-  lv_list_push(kp, w, sh, gcur, base, U);
+  __syncthreads();
   if (threadIdx.x == 0) stat_add(kp, &kp.stats->oversize, 1);
 }
 
@@ -362,8 +363,8 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
   int32_t* o = kp.o + P.o_base;
   int32_t* perm = kp.perm + P.perm_base;
   int32_t* btot = w.hist;          // [2][kMaxBlocks]: per-block child counts, parity by round
-  int32_t* gcur = w.sctl + 8;      // [2]: scratch cursors (children ids), parity by level
-  int32_t* scur = w.sctl + 10;     // [2]: oversize spill cursors, parity by level
+  int32_t* gcur = w.sctl + 8;      // [2]: overflow scratch cursors, parity by round
+  int32_t* scur = w.sctl + 10;     // [2]: oversize spill cursors, parity by round
   if (gtid() == 0) {
     place_root(kp, P, P.seed, P.pos0);
     gcur[0] = gcur[1] = scur[0] = scur[1] = 0;
@@ -380,11 +381,9 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
   auto tr = [&](int k, unsigned long long v) {
     if (kp.trace && b == 0 && threadIdx.x == 0 && nround < kp.trace_cap) kp.trace[(size_t)nround * kTraceW + k] = v;
   };
-  int lb = P.pos0, le = P.pos0 + 1, par = 0;
+  int lb = P.pos0, le = P.pos0 + 1, par = 0, rnd = 0;
   const int per_round = nb * kp.Bg;
   for (int level = 0;; ++level) {
-    int32_t* gc = gcur + (level & 1);
-    int32_t* sc = scur + (level & 1);
     int le_next = le;
     for (int rb = lb; rb < le; rb += per_round) {
       // ---- R: an even share of the round
@@ -392,14 +391,17 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       const int m = (re_ - rb + nb - 1) / nb;
       const int cb = min(re_, rb + b * m), ce = min(re_, cb + m);
       tr(0, globaltimer());
-      const int myc = lv_rediscover(kp, P, w, sm, sh, gc, sc, cb, ce - cb);
+      // the other parity's scratch was last allocated in round - 1 (before its
+      // barrier) and is read in W of round - 1: only its cursor is reset here,
+      // its space is reused after this round's barrier
+      if (gtid() == 0) { gcur[(rnd + 1) & 1] = 0; scur[(rnd + 1) & 1] = 0; }
+      const int myc = lv_rediscover(kp, P, w, sm, sh, gcur + (rnd & 1), scur + (rnd & 1), cb, ce - cb);
       if (threadIdx.x == 0) st_relaxed_s32(btot + par * kMaxBlocks + b, myc);
       tr(1, globaltimer());
       grid_barrier(kp);
       tr(2, globaltimer());
       tr(6, (unsigned long long)kp.ctl->dbg[7]);
       // ---- W: prefix of the block counts, output with fused reverse
-      if (gtid() == 0) { gcur[(level + 1) & 1] = 0; scur[(level + 1) & 1] = 0; }
       int total = 0, mx = 0;
       for (int i0 = 0; i0 < nb; i0 += kThreads) {
         const int i = i0 + threadIdx.x;
@@ -428,7 +430,7 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       int run = outn;
       for (int j = 0; j < sh.lv_n; ++j) {
         const int off = sh.lv_off[j], n = sh.lv_cnt[j];
-        for (int i = threadIdx.x; i < n; i += kThreads) put(run + i, __ldcg(w.vals1 + off + i));
+        for (int i = threadIdx.x; i < n; i += kThreads) put(run + i, __ldcg(lv_ovf(w) + off + i));
         run += n;
       }
       __syncthreads();
@@ -450,6 +452,7 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       le_next += total;
       par ^= 1;
       ++nround;
+      ++rnd;
     }
     grid_barrier(kp);
     if (nround > 0) { --nround; tr(5, globaltimer()); tr(7, (unsigned long long)kp.ctl->dbg[7]); ++nround; }
