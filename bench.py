@@ -121,14 +121,32 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def traffic_from_profile(key: str):
+def traffic_from_profile(key: str, field: str = "dram_bytes_per_launch"):
     p = os.path.join(ROOT, "profiles", f"traffic_{key}.json")
     if os.path.exists(p):
         try:
-            return json.load(open(p)).get("dram_bytes_per_launch")
+            return json.load(open(p)).get(field)
         except Exception:
             return None
     return None
+
+
+def _issue_roofline(dev, kern_ms: float, clocks: dict):
+    """Second bound of the C5 kernel (k_solo is issue/latency-bound, not HBM-bound):
+    warp instructions per launch (ncu smsp__inst_executed.sum of the same workload,
+    profiles/traffic_c5.json) / the live kernel time, against 4 issue slots per SM
+    per cycle x SMs x the SM clock sampled during the timed region."""
+    import torch
+    inst = traffic_from_profile("c5", "smsp_inst_executed_per_launch")
+    if not inst:
+        return None
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    mhz = (clocks or {}).get("sm_mhz") or (clocks or {}).get("sm_max_mhz") or 1965.0
+    peak = 4 * sms * mhz * 1e6 / 1e9   # G warp-instructions / s
+    ach = inst / (kern_ms * 1e-3) / 1e9
+    return {"bound": "issue", "achieved": round(ach, 1), "peak": round(peak, 1), "unit": "Gwarp-inst/s",
+            "frac": round(ach / peak, 4), "inst_per_launch": inst,
+            "note": "ncu instruction count of k_solo on this workload over the live kernel time"}
 
 
 def _plan_env() -> dict:
@@ -549,6 +567,7 @@ def run_c5(args, rank: int, world: int, local_rank: int, dist):
                      "peak_kind": peak_kind, "kernel": "k_solo (+ k_solo_order, 1 block)",
                      "algorithmic_bytes": alg_bytes, "csr_once_bytes": csr_once,
                      "csr_once_frac": round(csr_once / (km * 1e-3) / 1e9 / peak, 6)},
+        "issue_roofline": _issue_roofline(dev, km, clocks) if world == 1 else None,
         "cpu_baseline": {"value": round(o_nodes / o_sec / 1e6, 3), "unit": "Mnodes/s", "cores": cores,
                          "kind": "oracle", "ms": round(1e3 * o_sec, 1),
                          "sample": f"all {num} matrices ({o_nodes} nodes), serial oracle per matrix on a "
