@@ -507,6 +507,10 @@ def run_c5(args, rank: int, world: int, local_rank: int, dist):
                "h2d_bytes_per_step": 4 * (rp_h.numel() + ci_h.numel()) + 8 * 2 * (len(mine) + 1),
                "d2h_bytes_per_step": 4 * total, "ms_per_step": round(e2e_ms, 4), "steps": e2e_steps,
                "api": f"rcm_reorder_batched_host, {chunks} overlapped ranges"}
+        # the step is bound by the host link: H2D bytes over the step time
+        e2e["h2d_gbs"] = round(e2e["h2d_bytes_per_step"] / (e2e_ms * 1e-3) / 1e9, 2)
+        e2e["bound"] = ("host link (PCIe): the 11 GB CSR crosses it every step; the device "
+                        "ordering overlaps the copies of the next range")
         del rp_h, ci_h, perm_h
     except RuntimeError as ex:   # pinned host memory for ~11 GB may be unavailable
         e2e = {"value": None, "unit": "Mnodes/s", "unavailable": str(ex)[:120]}
