@@ -547,7 +547,10 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
   return level + 1;
 }
 
-static __device__ int gl_phase(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
+// Not inlined: with the warp-flattened BFS inlined, k_main<2,0>'s register
+// allocation moved spills into the chain's hot loop (ncu local-memory sectors
+// on C2 0.36 M -> 9.1 M; noinline: 4.2 M, C2 3.44 -> 3.40 ms, tools/gpu_spill.sh).
+static __device__ __noinline__ int gl_phase(const KParams& kp, const CompWS& w, int n, int r, ShState& sh) {
   int nl = gl_bfs(kp, w, n, r, sh);
   for (;;) {
     const int x = (int)(uint32_t)__ldcg(w.gkey);
