@@ -161,6 +161,25 @@ __device__ __forceinline__ int lv_ovf_reserve(const KParams& kp, const CompWS& w
   return base;
 }
 
+// Exclusive block scan with ONE barrier (warp totals in sh.wtmp32, read by
+// every warp after the barrier).  The caller guarantees a full barrier between
+// two calls (every R step has several), so one buffer suffices.
+__device__ __forceinline__ int lv_scan1(int v, ShState& sh, int& total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int x = warp_incl_scan(v);
+  if (lane == 31) sh.wtmp32[wid] = x;
+  __syncthreads();
+  int wv = lane < kWarps ? sh.wtmp32[lane] : 0;
+#pragma unroll
+  for (int d = 1; d < kWarps; d <<= 1) {
+    const int y = __shfl_up_sync(kFull, wv, d);
+    if (lane >= d) wv += y;
+  }
+  total = __shfl_sync(kFull, wv, kWarps - 1);
+  const int base = __shfl_sync(kFull, wv, (wid + 31) & 31);
+  return (wid ? base : 0) + x - v;
+}
+
 // The sorted, kept children of a batch (segments cand[p_eo[lp] .. + p_cnt[lp]))
 // in slot order, duplicates (adjacent after the sort) dropped: appended to the
 // block's shared-memory output buffer while it fits and no HBM entry exists
@@ -174,18 +193,18 @@ static __device__ void lv_emit(const KParams& kp, const CompWS& w, ShState& sh, 
     const int i = e - sm_p_eo(kp)[lp];
     return i < sm_p_cnt(kp)[lp] && (i == 0 || cand[e] != cand[e - 1]);
   };
+  // read before the scan's barrier; thread 0 updates lv_outn after it, and the
+  // caller's end-of-batch barrier orders that before the next batch's read
+  const int outn = sh.lv_outn, nlist = sh.lv_n;
   int k = 0;
   for (int e = b0; e < b1; ++e) k += valid(e);
   int tot;
-  int r = block_exclusive_scan<int32_t>(k, sh.wtmp32, tot);
+  int r = lv_scan1(k, sh, tot);
   if (tot == 0) return;
-  const int outn = sh.lv_outn;   // ids in the shared buffer (thread 0 updates it below, after the reads)
-  if (sh.lv_n == 0 && outn + tot <= kLvOut) {
+  if (nlist == 0 && outn + tot <= kLvOut) {
     for (int e = b0; e < b1; ++e)
       if (valid(e)) lv_out(kp)[outn + r++] = (int)(uint32_t)cand[e];
-    __syncthreads();
     if (threadIdx.x == 0) sh.lv_outn = outn + tot;
-    __syncthreads();
     return;
   }
   __syncthreads();
@@ -263,6 +282,37 @@ static __device__ void lv_oversize(const KParams& kp, const Problem& P, const Co
 // id, row start and valence in one round trip (o[], and prs / pdeg written by
 // D).  Cuts at T edge slots; sh.E = slots.
 static __device__ int lv_parents(const KParams& kp, const Problem& P, const CompWS& w, ShState& sh, int q0, int nP) {
+  if (nP <= kThreads) {   // one parent per thread: one-barrier scan, the T cut by a barrier count
+    const int t = threadIdx.x;
+    int rs = 0, d = 0;
+    if (t < nP) {
+      const int64_t x = P.o_base + q0 + t;
+      sm_p_v(kp)[t] = ld_cg_s32(kp.o + x);
+      rs = ld_cg_s32(w.front0 + x);
+      d = ld_cg_s32(w.front1 + x);
+    }
+    int E;
+    const int eo = lv_scan1(d, sh, E);
+    const bool fit = t < nP && (t == 0 || eo + d <= kp.T);   // the first parent always (oversize alone)
+    if (t < nP) {
+      sm_p_rs(kp)[t] = rs;
+      sm_p_eo(kp)[t] = eo;
+      sm_p_eo(kp)[t + 1] = eo + d;   // == the next parent's offset; the last one ends the slots
+      sm_p_cnt(kp)[t] = 0;
+    }
+    nP = __syncthreads_count(fit);
+    E = sm_p_eo(kp)[nP];
+    if (t == 0) { sh.nP = nP; sh.E = E; }
+    if (E <= kp.T) {
+      const int lane = t & 31;
+      for (int lp = t >> 5; lp < nP; lp += kWarps) {
+        const int eb = sm_p_eo(kp)[lp], ee = sm_p_eo(kp)[lp + 1];
+        for (int j = eb + lane; j < ee; j += 32) sm_lpof(kp)[j] = (uint16_t)lp;
+      }
+    }
+    __syncthreads();
+    return nP;
+  }
   for (int lp = threadIdx.x; lp < nP; lp += kThreads) {
     const int64_t x = P.o_base + q0 + lp;
     sm_p_v(kp)[lp] = ld_cg_s32(kp.o + x);
@@ -316,8 +366,10 @@ static __device__ int lv_rediscover(const KParams& kp, const Problem& P, const C
       __syncthreads();
       continue;
     }
-    for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm_p_cnt(kp)[lp] = 0;
-    __syncthreads();
+    if (min(kp.Bg, cnt - ob) > kThreads) {   // (the one-parent-per-thread load zeroed them)
+      for (int lp = threadIdx.x; lp < nP; lp += kThreads) sm_p_cnt(kp)[lp] = 0;
+      __syncthreads();
+    }
     // rediscovery (Alg. 5 ln 16-17): keep n iff owner(n) == key(p)
     const uint32_t kfirst = (uint32_t)(x0 + ob) + 1u;
     for (int e0 = threadIdx.x; e0 < E; e0 += kThreads * kDiscU) {
