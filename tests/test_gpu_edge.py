@@ -93,11 +93,12 @@ def test_duplicates_loops_unsorted_batched(rcm):
     assert np.array_equal(perm, ref)
 
 
+@pytest.mark.parametrize("path", ["default", "leveled"])
 @pytest.mark.parametrize("cfg", [1, 2, 3, 4])
-def test_pseudo_peripheral_full_configs(rcm, cfg):
+def test_pseudo_peripheral_full_configs(rcm, cfg, path):
     g, mode, start = synth.config_graph(cfg)
     ref = oracle.rcm(g.row_ptr, g.col_idx, oracle.PSEUDO_PERIPHERAL, 0)
-    got = _run(rcm, g, oracle.PSEUDO_PERIPHERAL, 0)
+    got = _run(rcm, g, oracle.PSEUDO_PERIPHERAL, 0, **PATHS[path])
     assert np.array_equal(got, ref)
 
 
