@@ -511,7 +511,8 @@ static __device__ int gl_bfs(const KParams& kp, const CompWS& w, int n, int r, S
       }
     }
     grid_barrier(kp);
-    const int nbig = ld_cg_s32(cbig + sl);
+    // items past a latched capacity error were never written: none are read then
+    const int nbig = ld_cg_s32(&kp.ctl->status) ? 0 : ld_cg_s32(cbig + sl);
     if (nbig) {   // uniform: read after the barrier
       for (int it = gwarp; it < nbig; it += nwarps) {
         const int p = __ldcg(w.vals0 + it), k = __ldcg(w.vals1 + it);

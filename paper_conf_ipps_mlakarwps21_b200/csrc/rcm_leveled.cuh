@@ -472,6 +472,7 @@ static __device__ void leveled_chain(const KParams& kp, const MainArgs& a, const
       const int xw = le_next + sh.written;
       auto put = [&](int i, int c) {
         const int x = xw + i;
+        if (x >= P.mat_n) { latch_error(kp.ctl, ST_CAPACITY); return; }   // only after a latched scratch error
         o[x] = c;
         perm[P.mat_n - 1 - x] = c;
         if (kp.iperm) kp.iperm[P.node_base + c] = P.mat_n - 1 - x;
