@@ -34,6 +34,7 @@
 // (same code, global atomics).  DESIGN.md §2.6.
 #pragma once
 #include "rcm_batch.cuh"
+#include "rcm_expand.cuh"
 
 // Read-only CSR loads: through the non-coherent path from HBM, or plain loads
 // when the whole CSR of a small graph was staged in shared memory (k_solo_sm).
@@ -410,18 +411,52 @@ __device__ __forceinline__ int so_deg(const SoloMat& M, int v) { return SO_LD(M.
 // the queue lives in the not-yet-written part of perm, visited bits in M.bvis.
 // Returns the number of levels; *minkey = min (valence, id) of the last level.
 static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long long* minkey, SoloSh& sh) {
+  constexpr int kU = 4;                       // edges per lane in flight
   int32_t* q = M.perm;                        // entries [0, n - written) are free
   so_zero_bits(M, M.bvis);
   __syncthreads();
   if (threadIdx.x == 0) { q[0] = r; so_claim_bit(M, M.bvis, r); sh.tail = 1; }
   __syncthreads();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   int head = 0, tail = 1, levels = 1;
   for (;;) {
-    for (int i = head + threadIdx.x; i < tail; i += kSoloNT) {
-      const int p = __ldcg(q + i);
-      for (int e = SO_LD(M.rp + p), ee = SO_LD(M.rp + p + 1); e < ee; ++e) {
-        const int c = SO_LD(M.col + e);
-        if (so_claim_bit(M, M.bvis, c)) q[atomicAdd(&sh.tail, 1)] = c;
+    // warp-cooperative expansion: a warp takes up to 32 frontier nodes and
+    // walks their rows as one flattened edge list (rcm_expand.cuh), kU column
+    // loads per lane in flight; new nodes appended with one atomic per warp
+    const int cnt = tail - head;
+    const int per = min(32, max(1, (cnt + kSoloNW - 1) / kSoloNW));
+    for (int i0 = wid * per; i0 < cnt; i0 += kSoloNW * per) {
+      int rs = 0, d = 0;
+      if (lane < per && i0 + lane < cnt) {
+        const int p = __ldcg(q + head + i0 + lane);
+        rs = SO_LD(M.rp + p);
+        d = SO_LD(M.rp + p + 1) - rs;
+      }
+      const int incl = warp_incl_scan(d), excl = incl - d;
+      const int E = __shfl_sync(kFull, incl, 31);
+      for (int b = 0; b < E; b += 32 * kU) {
+        int c[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+          const int e = b + u * 32 + lane;
+          const int jj = warp_edge_lane(e, incl) & 31;
+          const int r0 = __shfl_sync(kFull, rs, jj), x0 = __shfl_sync(kFull, excl, jj);
+          c[u] = e < E ? SO_LD(M.col + r0 + (e - x0)) : -1;
+        }
+        int k = 0;
+        bool nw[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) { nw[u] = c[u] >= 0 && so_claim_bit(M, M.bvis, c[u]); k += nw[u]; }
+        const int ki = warp_incl_scan(k);
+        const int kt = __shfl_sync(kFull, ki, 31);
+        if (kt) {
+          int base = 0;
+          if (lane == 31) base = atomicAdd(&sh.tail, kt);
+          base = __shfl_sync(kFull, base, 31) + ki - k;
+#pragma unroll
+          for (int u = 0; u < kU; ++u)
+            if (nw[u]) q[base++] = c[u];
+        }
       }
     }
     __syncthreads();
@@ -444,7 +479,8 @@ static __device__ int so_bfs(const SoloMat& M, int written, int r, unsigned long
 
 // GL finder (C-5): BFS from r, next root = min (valence, id) of the
 // last level, repeat while the level count grows, return the last root.
-static __device__ int so_gl(const SoloMat& M, int written, int r, SoloSh& sh) {
+// Not inlined: keeps the warp-flattened BFS out of k_solo's register allocation.
+static __device__ __noinline__ int so_gl(const SoloMat& M, int written, int r, SoloSh& sh) {
   unsigned long long key;
   int nl = so_bfs(M, written, r, &key, sh);
   int x = (int)(uint32_t)key;
