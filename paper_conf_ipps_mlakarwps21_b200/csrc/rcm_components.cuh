@@ -315,36 +315,66 @@ static __device__ void cc_phase(const KParams& kp, const MainArgs& a, const Smem
   chunk_of(kp, n, cb, ce);
   {
     int cnt = 0;
+    // isolated nodes (valence 0, C-2) are components of their own whose C-6 key
+    // (0, id) precedes every other: they take the first positions in id order
+    // directly and stay out of the sort (C4: 2.18 M of its 2.19 M components)
+    int iso = 0;
     for (long long v = cb + threadIdx.x; v < ce; v += kThreads) {
       const int r = __ldcg(w.label + v);
-      cnt += (r >= 0 && (int)(uint32_t)__ldcg(w.ckey + r) == (int)v);
+      if (r >= 0) {
+        const unsigned long long k = __ldcg(w.ckey + r);
+        const bool rep = (int)(uint32_t)k == (int)v;
+        cnt += rep && (k >> 32) != 0;
+        iso += rep && (k >> 32) == 0;
+      }
     }
     cnt = block_reduce_sum<int32_t>(cnt, sh.wtmp32);
-    if (threadIdx.x == 0) w.hist[blockIdx.x] = cnt;
+    iso = block_reduce_sum<int32_t>(iso, sh.wtmp32);
+    if (threadIdx.x == 0) { w.hist[blockIdx.x] = cnt; w.hist[2 * kp.nblocks + blockIdx.x] = iso; }
   }
   grid_barrier(kp);
   if (blockIdx.x == 0) {
     const int tot = block_scan_partials<int32_t>(w.hist, w.hist + kp.nblocks, kp.nblocks, sh.wtmp32);
-    if (threadIdx.x == 0) { w.sctl[0] = tot; w.sctl[1] = 0; }
+    const int niso = block_scan_partials<int32_t>(w.hist + 2 * kp.nblocks, w.hist + 3 * kp.nblocks, kp.nblocks,
+                                                  sh.wtmp32);
+    if (threadIdx.x == 0) { w.sctl[0] = tot; w.sctl[1] = 0; w.sctl[4] = niso; }
   }
   grid_barrier(kp);
   {
     int run = __ldcg(w.hist + kp.nblocks + blockIdx.x);
+    int irun = ld_cg_s32(&kp.ctl->chain_total) + __ldcg(w.hist + 3 * kp.nblocks + blockIdx.x);
     for (long long base = cb; base < ce; base += kThreads) {
       const long long v = base + threadIdx.x;
-      int r = -1, f = 0;
+      int r = -1, f = 0, fi = 0;
       unsigned long long k = 0;
       if (v < ce) {
         r = __ldcg(w.label + v);
-        if (r >= 0) { k = __ldcg(w.ckey + r); f = (int)(uint32_t)k == (int)v; }
+        if (r >= 0) {
+          k = __ldcg(w.ckey + r);
+          const bool rep = (int)(uint32_t)k == (int)v;
+          f = rep && (k >> 32) != 0;
+          fi = rep && (k >> 32) == 0;
+        }
       }
-      int tot;
+      int tot, itot;
       const int ex = block_exclusive_scan<int32_t>(f, sh.wtmp32, tot);
+      const int iex = block_exclusive_scan<int32_t>(fi, sh.wtmp32, itot);
       if (f) {
         w.keys0[run + ex] = ((k >> 32) << a.idbits) | (k & 0xffffffffull);
         w.vals0[run + ex] = r;
       }
+      if (fi) {   // an isolated node: its position now
+        const int pos = irun + iex;
+        kp.o[pos] = (int)v;
+        kp.perm[n - 1 - pos] = (int)v;
+        if (kp.iperm) kp.iperm[v] = n - 1 - pos;
+      }
       run += tot;
+      irun += itot;
+    }
+    if (kp.collect_stats) {
+      const int mine = __ldcg(w.hist + 2 * kp.nblocks + blockIdx.x);
+      if (threadIdx.x == 0 && mine) atomicAdd(&kp.stats->components, (unsigned long long)mine);
     }
   }
   grid_barrier(kp);
@@ -381,7 +411,7 @@ static __device__ void cc_phase(const KParams& kp, const MainArgs& a, const Smem
   Problem* solos = const_cast<Problem*>(kp.solos);
   int singles = 0;
   {
-    long long run = (long long)ld_cg_s32(&kp.ctl->chain_total) + __ldcg(w.hist + blockIdx.x);
+    long long run = (long long)ld_cg_s32(&kp.ctl->chain_total) + ld_cg_s32(w.sctl + 4) + __ldcg(w.hist + blockIdx.x);
     for (long long base = cb; base < ce; base += kThreads) {
       const long long i = base + threadIdx.x;
       int root = -1, size = 0;
