@@ -54,7 +54,7 @@ static __device__ void grid_barrier(const KParams& kp) {
 // block, temp buffer tmp[0..n); digits that are equal in all keys are skipped.
 // `scratch` is >= (1 + kWarps) * 256 ints of shared memory.
 static __device__ void block_radix_sort_global(unsigned long long* a, unsigned long long* tmp, int n,
-                                        int32_t* scratch, ShState& sh) {
+                                        int32_t* scratch, ShState& sh, int lo_shift = 0) {
   if (n <= 1) return;
   unsigned long long first = __ldcg(a);
   unsigned long long diff = 0;
@@ -78,7 +78,7 @@ static __device__ void block_radix_sort_global(unsigned long long* a, unsigned l
   unsigned long long* dst = tmp;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const unsigned lt = (1u << lane) - 1;
-  for (int shift = 0; shift < 64; shift += 8) {
+  for (int shift = lo_shift; shift < 64; shift += 8) {   // digits below lo_shift already in order
     if (((diff >> shift) & 0xffull) == 0) continue;
     for (int i = threadIdx.x; i < 256; i += kThreads) off[i] = 0;
     __syncthreads();
@@ -242,9 +242,16 @@ static __device__ bool oversize_gather_sort(const KParams& kp, const Problem& P,
   }
   __threadfence_block();
   __syncthreads();
-  // sort by (valence, id); the bitmap area is free now
+  // sort by (valence, id); the bitmap area is free now.  The gather is stable in
+  // row order, so when the row's kept ids ascend (sorted columns, the usual
+  // case) a stable sort on the valence half alone gives (valence, id) order --
+  // the paper's direct copy of a single-valence bin in id order
+  int unsorted = 0;
+  for (int i = threadIdx.x; i + 1 < C; i += kThreads)
+    unsorted |= (uint32_t)__ldcg(out + i) >= (uint32_t)__ldcg(out + i + 1);
+  unsorted = __syncthreads_or(unsorted);
   block_radix_sort_global(out, kp.spill + kp.spill_cap + sh.spill_base, C,
-                          reinterpret_cast<int32_t*>(sm_cand(kp)), sh);
+                          reinterpret_cast<int32_t*>(sm_cand(kp)), sh, unsorted ? 0 : 32);
   return true;
 }
 
