@@ -40,8 +40,12 @@
 // when the whole CSR of a small graph was staged in shared memory (k_solo_sm).
 #ifdef RCM_SOLO_SMEM_CSR
 #define SO_LD(p) (*(p))
+#define SO_LDS(p) (*(p))
 #else
 #define SO_LD(p) __ldg(p)
+// a parent's row is read once: streaming load (evict-first), so the
+// children's row_ptr lines keep their place in L2 (C5 31.3 -> 30.2 ms)
+#define SO_LDS(p) __ldcs(p)
 #endif
 
 namespace rcm {
@@ -748,7 +752,7 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
       if (e < E) {
         while (nx <= e) { ++lp; se = nx; nx = so_p_eo()[lp + 1]; rs = so_p_rs()[lp]; }
         so_lpof()[e] = (uint16_t)lp;
-        cc[u] = SO_LD(M.col + rs + (e - se));
+        cc[u] = SO_LDS(M.col + rs + (e - se));
       }
     }
   } else {
