@@ -319,3 +319,22 @@ def test_batched_host_pipeline(rcm, chunks):
         assert rcm.rcm_sync_status(plan.handle) == 0
         assert np.array_equal(perm_h.numpy(), ref), (mode, chunks)
     plan.close()
+
+
+@pytest.mark.parametrize("path", ["default", "chain", "leveled"])
+def test_isolated_nodes(rcm, path):
+    """Isolated nodes (valence 0) take the first component positions in id
+    order directly (components phase fast path, C-6): an edgeless graph, and
+    isolated nodes interleaved with grids, stars and paths under a relabelling,
+    for FIXED (a non-isolated start), MIN_DEGREE and PSEUDO_PERIPHERAL."""
+    empty = synth.csr_from_pairs(1000, np.zeros(0, np.int64), np.zeros(0, np.int64))
+    parts = [synth.grid2d(15, 9), synth.path(1), synth.star(25), synth.path(1), synth.path(1),
+             synth.relabel(synth.grid3d_27(5, 5, 4), synth.randperm(100, 7)), synth.path(1), synth.path(9)]
+    mixed = synth.relabel(synth.disjoint_union(parts), synth.randperm(sum(p.n for p in parts), 8))
+    for g in (empty, mixed):
+        starts = [(oracle.MIN_DEGREE, 0), (oracle.PSEUDO_PERIPHERAL, 0)]
+        if g.nnz:
+            starts.append((oracle.FIXED, int(np.argmax(np.diff(g.row_ptr)))))
+        for mode, s0 in starts:
+            ref = oracle.rcm(g.row_ptr, g.col_idx, mode, s0)
+            assert np.array_equal(_run(rcm, g, mode, s0, **PATHS[path]), ref), (g.n, mode)
