@@ -701,8 +701,8 @@ static __device__ void so_step(const SoloArgs& a, const SoloMat& M, SoloSh& sh, 
     const int lo = kBig ? S.pos : rhi;
     const int hi = min(S.written, S.pos + kSoloQ);
     for (int q = lo + t; q < hi; q += kSoloNT) {
-      const int v = __ldcg(M.perm + last - q);
-      int2 rd = (kBig || !kSoloPend) ? make_int2(0, -1) : __ldcg(a.pend + M.node_base + q);   // coalesced
+      const int v = __ldcs(M.perm + last - q);   // read once (streaming)
+      int2 rd = (kBig || !kSoloPend) ? make_int2(0, -1) : __ldcs(a.pend + M.node_base + q);   // coalesced
       if (rd.y < 0) { rd.x = SO_LD(M.rp + v); rd.y = SO_LD(M.rp + v + 1) - rd.x; }
       so_ring_v()[q & (kSoloQ - 1)] = v;
       so_ring_rs()[q & (kSoloQ - 1)] = rd.x;
